@@ -1,0 +1,222 @@
+/*
+ * nest.h -- C ABI of the B200 three-level (teams -> parallel -> simd) loop-nest
+ * library.  ABI v1.
+ *
+ * What it executes (PAPER.md = /root/reference/PAPER.md, Wright et al.,
+ * "Implementing OpenMP's SIMD Directive in LLVM's GPU Runtime", ICPP'23):
+ *   - teams    -> thread blocks ("league of teams")
+ *   - parallel -> SIMD groups of `simdlen` adjacent lanes inside one warp
+ *                 (getSimdGroup/Id/Size, isSimdGroupLeader,
+ *                 simdmask: PAPER.md:507-529)
+ *   - simd     -> the lanes of a group, cyclic worksharing iv = id, id+S, ...
+ *                 (Fig 8)
+ * in one of the two execution models of the parallel region:
+ *   - SPMD (GPU-centric): every lane runs the sequential
+ *     code redundantly, side effects guarded to the SIMD main;
+ *   - generic (CPU-centric, Figs 3/4/6): only the SIMD
+ *     main runs the sequential code; before each simd loop it posts
+ *     {fn, trip count, loop state} to its group and releases the workers with
+ *     a warp-level barrier; a null fn terminates.  The state travels through
+ *     the group's slot of a shared-memory "variable sharing space"
+ *     (2048 B per team by default, split evenly, global
+ *     fallback when it does not fit) -- NEST_MODE_GENERIC_SMEM -- or through
+ *     warp shuffles from the main -- NEST_MODE_GENERIC_SHFL (north_star).
+ * Each simd loop ends with a reduction across the group's lanes by a
+ * __shfl_xor_sync butterfly (north_star addition: the paper has no reduction,
+ * PAPER.md:868-873, 880-884).  simdlen = 1 is the flat two-level mapping
+ * (simd folded into threads).
+ *
+ * Conventions for every entry point:
+ *   - Array arguments are DEVICE pointers owned by the caller (except the
+ *     *_hostio call, whose data arguments are HOST pointers).  `stream` is a
+ *     cudaStream_t passed as void* (NULL = legacy default stream).
+ *   - Calls are asynchronous and stream-ordered; they never synchronise the
+ *     device except where stated.  Device faults surface at the caller's
+ *     next synchronisation.
+ *   - All validation happens BEFORE any launch; a non-OK status means nothing
+ *     was enqueued.  Zero-size problems return NEST_OK without a launch.
+ *   - nest_last_error() returns a thread-local description of the last
+ *     non-OK status.  Nothing throws across the ABI.
+ *   - Preconditions that are documented but not checked in the hot path:
+ *     rowptr monotone with rowptr[0] == 0 and rowptr[nrows] == nnz,
+ *     0 <= colind < ncols; pointers suitably aligned for their type.
+ *     nest_csr_validate() checks the CSR ones on the device.
+ *   - The library allocates nothing per call.  Library-owned lazily-grown
+ *     device scratch (the sharing-space global fallback)
+ *     is released by nest_shutdown().
+ */
+#ifndef NEST_H
+#define NEST_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define NEST_ABI_VERSION 1u
+
+typedef enum {
+    NEST_OK = 0,
+    NEST_ERR_INVALID_ARG = 1,   /* bad extent, simdlen, team size, null pointer ... */
+    NEST_ERR_UNSUPPORTED = 2,   /* valid but not built (e.g. T above the kernel's limit) */
+    NEST_ERR_CUDA = 3,          /* a CUDA runtime call failed (no device, launch error) */
+    NEST_ERR_NCCL = 4,
+    NEST_ERR_NO_MEMORY = 5
+} nest_status;
+
+/* Execution model of the parallel region. */
+typedef enum {
+    NEST_MODE_SPMD = 0,          /* all lanes run everything; no communication */
+    NEST_MODE_GENERIC_SMEM = 1,  /* main posts loop state in the shared sharing space */
+    NEST_MODE_GENERIC_SHFL = 2   /* main broadcasts loop state with warp shuffles */
+} nest_mode;
+
+/* Reduction of the simd loop (identity +0.0 / -inf / +inf). */
+typedef enum { NEST_REDUCE_SUM = 0, NEST_REDUCE_MAX = 1, NEST_REDUCE_MIN = 2 } nest_reduce;
+
+/* flags */
+enum {
+    /* grid = min(needed, resident blocks) and teams stride over the outer
+     * loop ("teams distribute" with a persistent league).  Implied when the
+     * sharing space falls back to global memory. */
+    NEST_F_PERSISTENT_GRID = 1u << 0,
+    /* stream the CSR arrays with L2 evict-first / L1 no-allocate hints and
+     * keep x cached (SpMV only; results unchanged). */
+    NEST_F_STREAM_HINTS = 1u << 1
+};
+
+/* The nest descriptor: team, thread and simd extents, mode and reduction.
+ * Zero-initialise, set abi_version = NEST_ABI_VERSION, then override. */
+typedef struct {
+    uint32_t abi_version;       /* == NEST_ABI_VERSION */
+    int32_t num_teams;          /* grid size; 0 = auto (see nest_plan) */
+    int32_t threads_per_team;   /* T: multiple of 32 in [32, 1024]; 0 = 256 */
+    int32_t simdlen;            /* S: SIMD group size 1, 2, 4, 8, 16 or 32 */
+    int32_t mode;               /* nest_mode */
+    int32_t reduce;             /* nest_reduce */
+    int32_t sharing_bytes;      /* generic sharing space per team; 0 = 2048 */
+    uint32_t flags;             /* NEST_F_* */
+    int32_t outer_unroll;       /* U: outer iterations a group keeps in flight (1, 2, 4); 0 = 1 */
+    int32_t x_halo;             /* SpMV only. > 0: stage x in shared memory as a sliding window
+                                 * [row0 - x_halo, row0 + rows + x_halo) around each team's chunk of
+                                 * rows (banded matrices); columns outside it read global memory.
+                                 * Results are identical; 0 = no staging. */
+    int32_t reserved[2];        /* must be 0 */
+} nest_desc;
+
+/* Resolved launch geometry (a1). */
+typedef struct {
+    int32_t grid;                 /* teams (blocks) */
+    int32_t block;                /* threads per team T */
+    int32_t groups_per_team;      /* G = T / S */
+    int32_t slot_bytes;           /* sharing_bytes / G (generic-SMEM slot per group) */
+    int32_t payload_bytes;        /* bytes one group posts per simd batch */
+    int32_t uses_global_fallback; /* payload_bytes > slot_bytes (GENERIC_SMEM only) */
+    int32_t outer_unroll;         /* U */
+    int32_t smem_bytes;           /* dynamic shared memory per team */
+} nest_plan_info;
+
+uint32_t nest_abi_version(void);
+const char *nest_status_str(nest_status s);
+const char *nest_last_error(void);
+
+/* a1: validate `desc` and resolve the geometry for `outer_iters` outer
+ * iterations whose generic payload is `payload_bytes` per group.  Host-only
+ * unless the grid must be sized from device occupancy (num_teams == 0 with
+ * NEST_F_PERSISTENT_GRID or a global fallback), which queries the current
+ * device (NEST_ERR_CUDA without one).  Errors: NEST_ERR_INVALID_ARG. */
+nest_status nest_plan(const nest_desc *desc, int64_t outer_iters, int32_t payload_bytes,
+                      nest_plan_info *out);
+
+/* a8: CSR SpMV, y[i] = (+)_{k in [rowptr[i], rowptr[i+1])} val[k] * x[colind[k]]
+ * (sparse_matvec).  Outer (parallel) unit = a row; simd
+ * unit = a nonzero of the row.  rowptr int64[nrows+1], colind int32[nnz],
+ * val f64[nnz], x f64[ncols], y f64[nrows] (written).  nrows, ncols, nnz >= 0. */
+nest_status nest_spmv_csr_f64(const nest_desc *desc, int64_t nrows, int64_t ncols, int64_t nnz,
+                              const int64_t *rowptr, const int32_t *colind, const double *val,
+                              const double *x, double *y, void *stream);
+
+/* a8 end to end from HOST buffers (pinned for asynchronous copies): copies
+ * rowptr/colind/val/x into `d_workspace` (device, >= nest_spmv_hostio_workspace_bytes),
+ * runs nest_spmv_csr_f64 and copies y back into h_y, all on `stream`.  The
+ * host buffers must stay valid until the stream reaches that point. */
+size_t nest_spmv_hostio_workspace_bytes(int64_t nrows, int64_t ncols, int64_t nnz);
+nest_status nest_spmv_csr_f64_hostio(const nest_desc *desc, int64_t nrows, int64_t ncols,
+                                     int64_t nnz, const int64_t *h_rowptr,
+                                     const int32_t *h_colind, const double *h_val,
+                                     const double *h_x, double *h_y, void *d_workspace,
+                                     size_t workspace_bytes, void *stream);
+
+/* a9: batched small dense matvec (SU3_bench stand-in):
+ * y[b][r] = (+)_{k<n} A[b][r][k] * x[b][k], fp32.  Outer unit = a batch b;
+ * the parallel region runs r = 0..m-1 sequentially, one simd loop over k each.
+ * A f32[batch][m][n] row-major, x f32[batch][n], y f32[batch][m]. */
+nest_status nest_batched_matvec_f32(const nest_desc *desc, int64_t batch, int32_t m, int32_t n,
+                                    const float *A, const float *x, float *y, void *stream);
+
+/* a10: nested loop with a sequential prologue ("benchmark kernel" stand-in,
+ * PAPER.md:900-907; generic-vs-SPMD study PAPER.md:944-972).  For each outer i:
+ *   scale = w[i]; base = 1 + i*L; visits += 1 (guarded: once per i in every mode);
+ *   trip = scale == 0 ? 0 : L;
+ *   s = (+)_{j<trip} coef[j] * ((in[base+j-1] + 2*in[base+j]) + in[base+j+1]);
+ *   out[i] = trip == 0 ? +0.0 : scale * s.
+ * in f64[nouter*L+2], coef f64[L], w f64[nouter], out f64[nouter];
+ * visits: one u64 accumulated into (may be NULL). */
+nest_status nest_nested_stencil_f64(const nest_desc *desc, int64_t nouter, int32_t L,
+                                    const double *in, const double *coef, const double *w,
+                                    double *out, unsigned long long *visits, void *stream);
+
+/* a2/a5/a6 probe.  out_map int32[grid*block*5] (may be NULL): per thread
+ * {getSimdGroup, getSimdGroupId, getSimdGroupSize, isSimdGroupLeader, simdmask}
+ * (PAPER.md:507-529).  Then one outer iteration per group (outer = grid*G)
+ * runs one simd loop of `trip` iterations through the selected mode engine:
+ * hits int32[trip] (zeroed by the caller, may be NULL) receives one atomic
+ * increment per group per iteration; owner int32[trip] (may be NULL) receives
+ * the lane id that ran iteration j in global group 0 (Fig 8); totals
+ * f64[grid*G] (may be NULL) receives each group's reduced count of executed
+ * iterations (== trip under SUM).  num_teams must be > 0. */
+nest_status nest_probe_mapping(const nest_desc *desc, int32_t *out_map, int64_t trip,
+                               int32_t *hits, int32_t *owner, double *totals, void *stream);
+
+/* Debug: check CSR preconditions on the device.  *d_bad (device int32, zeroed
+ * by the caller) receives a nonzero value if rowptr is not monotone, does not
+ * start at 0 / end at nnz, or a column index is out of range. */
+nest_status nest_csr_validate(int64_t nrows, int64_t ncols, int64_t nnz, const int64_t *rowptr,
+                              const int32_t *colind, int32_t *d_bad, void *stream);
+
+/* Bench utility: overwrite `bytes` of device memory at `buf` (flushes L2). */
+nest_status nest_util_l2_flush(void *buf, size_t bytes, void *stream);
+
+/* ---- a12: row-partitioned multi-GPU SpMV (north_star; the paper is single-GPU) ----
+ * One process per GPU.  Rank r owns rows [r*chunk, min((r+1)*chunk, n)) and the
+ * same slice of x, chunk = ceil(n / nranks).  Each call all-gathers x over NCCL
+ * (NVLink) into x_full (nranks*chunk doubles, so global column j is x_full[j])
+ * and runs the local SpMV on the same stream. */
+typedef struct nest_comm nest_comm;
+
+/* 128-byte NCCL unique id, created on one rank and broadcast by the caller. */
+nest_status nest_comm_unique_id(uint8_t out[128]);
+/* Collective: every rank calls with the same id; binds the current device. */
+nest_status nest_comm_init(const uint8_t id[128], int32_t nranks, int32_t rank, nest_comm **out);
+nest_status nest_comm_destroy(nest_comm *comm);
+/* Rows: chunk = ceil(nrows_global / nranks), this rank's nrows_local rows start at
+ * rank*chunk; rowptr_local is 0-based for them and colind holds GLOBAL column
+ * indices.  x: xchunk = ceil(ncols_global / nranks); x_local holds xchunk doubles
+ * (entries past ncols_global on the tail rank are ignored); x_full receives
+ * nranks*xchunk doubles, so global column j is x_full[j]. */
+nest_status nest_spmv_csr_f64_dist(const nest_desc *desc, nest_comm *comm, int64_t nrows_global,
+                                   int64_t ncols_global, int64_t nrows_local, int64_t nnz_local,
+                                   const int64_t *rowptr_local, const int32_t *colind,
+                                   const double *val, const double *x_local, double *x_full,
+                                   double *y_local, void *stream);
+
+/* Release library-owned device scratch of the current device. */
+nest_status nest_shutdown(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* NEST_H */

@@ -1,0 +1,77 @@
+"""ctypes binding of libnest.so (include/nest.h), argument marshalling only.
+
+Every C entry point is exposed under its own name (``nest_spmv_csr_f64`` ...)
+with its C signature; the friendlier wrappers in ``api.py`` accept torch
+tensors and turn a non-OK status into ``NestError``.  There is no fallback:
+if libnest.so is missing or fails to load, importing this module raises.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libnest.so")
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(f"{LIB_PATH} is missing: build it with `make -C {os.path.dirname(_HERE)}` "
+                      "(there is no CPU fallback)")
+lib = ctypes.CDLL(LIB_PATH)
+
+NEST_ABI_VERSION = 1
+NEST_OK, NEST_ERR_INVALID_ARG, NEST_ERR_UNSUPPORTED, NEST_ERR_CUDA, NEST_ERR_NCCL, NEST_ERR_NO_MEMORY = range(6)
+NEST_MODE_SPMD, NEST_MODE_GENERIC_SMEM, NEST_MODE_GENERIC_SHFL = 0, 1, 2
+NEST_REDUCE_SUM, NEST_REDUCE_MAX, NEST_REDUCE_MIN = 0, 1, 2
+NEST_F_PERSISTENT_GRID = 1 << 0
+NEST_F_STREAM_HINTS = 1 << 1
+
+
+class nest_desc(ctypes.Structure):
+    _fields_ = [("abi_version", ctypes.c_uint32), ("num_teams", ctypes.c_int32),
+                ("threads_per_team", ctypes.c_int32), ("simdlen", ctypes.c_int32),
+                ("mode", ctypes.c_int32), ("reduce", ctypes.c_int32),
+                ("sharing_bytes", ctypes.c_int32), ("flags", ctypes.c_uint32),
+                ("outer_unroll", ctypes.c_int32), ("x_halo", ctypes.c_int32),
+                ("reserved", ctypes.c_int32 * 2)]
+
+
+class nest_plan_info(ctypes.Structure):
+    _fields_ = [("grid", ctypes.c_int32), ("block", ctypes.c_int32),
+                ("groups_per_team", ctypes.c_int32), ("slot_bytes", ctypes.c_int32),
+                ("payload_bytes", ctypes.c_int32), ("uses_global_fallback", ctypes.c_int32),
+                ("outer_unroll", ctypes.c_int32), ("smem_bytes", ctypes.c_int32)]
+
+
+_i32, _i64, _u32, _vp, _sz = ctypes.c_int32, ctypes.c_int64, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_size_t
+_st = ctypes.c_int
+_D = ctypes.POINTER(nest_desc)
+
+# name -> (restype, argtypes); every symbol include/nest.h declares
+SIGNATURES = {
+    "nest_abi_version": (_u32, []),
+    "nest_status_str": (ctypes.c_char_p, [_st]),
+    "nest_last_error": (ctypes.c_char_p, []),
+    "nest_plan": (_st, [_D, _i64, _i32, ctypes.POINTER(nest_plan_info)]),
+    "nest_spmv_csr_f64": (_st, [_D, _i64, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp]),
+    "nest_spmv_hostio_workspace_bytes": (_sz, [_i64, _i64, _i64]),
+    "nest_spmv_csr_f64_hostio": (_st, [_D, _i64, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _sz, _vp]),
+    "nest_batched_matvec_f32": (_st, [_D, _i64, _i32, _i32, _vp, _vp, _vp, _vp]),
+    "nest_nested_stencil_f64": (_st, [_D, _i64, _i32, _vp, _vp, _vp, _vp, _vp, _vp]),
+    "nest_probe_mapping": (_st, [_D, _vp, _i64, _vp, _vp, _vp, _vp]),
+    "nest_csr_validate": (_st, [_i64, _i64, _i64, _vp, _vp, _vp, _vp]),
+    "nest_util_l2_flush": (_st, [_vp, _sz, _vp]),
+    "nest_comm_unique_id": (_st, [_vp]),
+    "nest_comm_init": (_st, [_vp, _i32, _i32, ctypes.POINTER(_vp)]),
+    "nest_comm_destroy": (_st, [_vp]),
+    "nest_spmv_csr_f64_dist": (_st, [_D, _vp, _i64, _i64, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _vp]),
+    "nest_shutdown": (_st, []),
+}
+
+for _name, (_res, _args) in SIGNATURES.items():
+    _f = getattr(lib, _name)
+    _f.restype = _res
+    _f.argtypes = _args
+    globals()[_name] = _f
+
+if lib.nest_abi_version() != NEST_ABI_VERSION:
+    raise ImportError(f"libnest.so ABI {lib.nest_abi_version()} != {NEST_ABI_VERSION}")

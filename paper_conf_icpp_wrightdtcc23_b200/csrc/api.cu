@@ -1,0 +1,421 @@
+// api.cu -- the C ABI of include/nest.h: validation, the a1 planner, the
+// library-owned sharing-space fallback and the single-GPU entry points.
+#include <cuda_runtime.h>
+
+#include <climits>
+#include <cstdarg>
+#include <cstdio>
+#include <mutex>
+
+#include "internal.h"
+
+namespace nest {
+
+static thread_local char g_err[512] = "";
+
+nest_status fail(nest_status s, const char* fmt, ...) {
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(g_err, sizeof(g_err), fmt, ap);
+    va_end(ap);
+    return s;
+}
+
+nest_status cuda_fail(cudaError_t e, const char* what) {
+    cudaGetLastError();   // clear a sticky-free error so the next call starts clean
+    return fail(NEST_ERR_CUDA, "%s: %s (%s)", what, cudaGetErrorName(e), cudaGetErrorString(e));
+}
+
+static nest_status sm_count(int* out) {
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
+    e = cudaDeviceGetAttribute(out, cudaDevAttrMultiProcessorCount, dev);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaDeviceGetAttribute(SM count)");
+    return NEST_OK;
+}
+
+static bool valid_simdlen(int32_t s) {
+    return s == 1 || s == 2 || s == 4 || s == 8 || s == 16 || s == 32;
+}
+
+static constexpr int32_t kDefaultThreads = 256;
+static constexpr int32_t kDefaultSharing = 2048;
+static constexpr int32_t kMaxSharing = 48 * 1024;       // static-carveout dynamic smem
+static constexpr int32_t kMaxBlocksPerSm = 32;
+static constexpr int32_t kMaxThreadsPerSm = 2048;
+static constexpr int32_t kSmemPerSm = 228 * 1024;
+static constexpr int32_t kSmemReservedPerBlock = 1024;
+static constexpr int32_t kMaxDynSmem = 227 * 1024;
+
+// Descriptor validation (groups are equal,
+// inside one warp, and divide the team evenly).
+static nest_status validate_desc(const nest_desc* d, int32_t* T, int32_t* sharing, int32_t* U) {
+    if (!d) return fail(NEST_ERR_INVALID_ARG, "desc is NULL");
+    if (d->abi_version != NEST_ABI_VERSION)
+        return fail(NEST_ERR_INVALID_ARG, "abi_version %u != %u", d->abi_version, NEST_ABI_VERSION);
+    *T = d->threads_per_team ? d->threads_per_team : kDefaultThreads;
+    if (*T < 32 || *T > 1024 || *T % 32)
+        return fail(NEST_ERR_INVALID_ARG, "threads_per_team %d: need a multiple of 32 in [32,1024]", *T);
+    if (!valid_simdlen(d->simdlen))
+        return fail(NEST_ERR_INVALID_ARG, "simdlen %d: need 1, 2, 4, 8, 16 or 32", d->simdlen);
+    if (d->mode < NEST_MODE_SPMD || d->mode > NEST_MODE_GENERIC_SHFL)
+        return fail(NEST_ERR_INVALID_ARG, "mode %d", d->mode);
+    if (d->reduce < NEST_REDUCE_SUM || d->reduce > NEST_REDUCE_MIN)
+        return fail(NEST_ERR_INVALID_ARG, "reduce %d", d->reduce);
+    *sharing = d->sharing_bytes ? d->sharing_bytes : kDefaultSharing;
+    if (*sharing < 0 || *sharing > kMaxSharing)
+        return fail(NEST_ERR_INVALID_ARG, "sharing_bytes %d: need [0, %d]", d->sharing_bytes, kMaxSharing);
+    if (d->num_teams < 0) return fail(NEST_ERR_INVALID_ARG, "num_teams %d < 0", d->num_teams);
+    *U = d->outer_unroll ? d->outer_unroll : 1;
+    if (*U != 1 && *U != 2 && *U != 4)
+        return fail(NEST_ERR_INVALID_ARG, "outer_unroll %d: need 1, 2 or 4", d->outer_unroll);
+    if (d->flags & ~(uint32_t)(NEST_F_PERSISTENT_GRID | NEST_F_STREAM_HINTS))
+        return fail(NEST_ERR_INVALID_ARG, "unknown flags 0x%x", d->flags);
+    if (d->reserved[0] || d->reserved[1])
+        return fail(NEST_ERR_INVALID_ARG, "reserved fields must be 0");
+    return NEST_OK;
+}
+
+static nest_status resident_blocks(int32_t T, int32_t smem, int64_t* out) {
+    int sms = 0;
+    nest_status s = sm_count(&sms);
+    if (s != NEST_OK) return s;
+    int32_t per_sm = kMaxBlocksPerSm;
+    if (kMaxThreadsPerSm / T < per_sm) per_sm = kMaxThreadsPerSm / T;
+    if (smem > 0) {
+        const int32_t by_smem = kSmemPerSm / (smem + kSmemReservedPerBlock);
+        if (by_smem < per_sm) per_sm = by_smem;
+    }
+    *out = (int64_t)sms * (per_sm > 0 ? per_sm : 1);
+    return NEST_OK;
+}
+
+static nest_status plan_core(const nest_desc* d, int64_t outer, int32_t K, int32_t T,
+                             int32_t sharing, int32_t U, int32_t payload, Plan* p, bool spmv_window) {
+    if (outer < 0) return fail(NEST_ERR_INVALID_ARG, "outer iterations %lld < 0", (long long)outer);
+    if (d->x_halo < 0) return fail(NEST_ERR_INVALID_ARG, "x_halo %d < 0", d->x_halo);
+    if (d->x_halo > 0 && !spmv_window)
+        return fail(NEST_ERR_INVALID_ARG, "x_halo applies to the CSR SpMV only");
+    if (K <= 0) K = 1;
+    const int32_t S = d->simdlen;
+    const bool smem_mode = d->mode == NEST_MODE_GENERIC_SMEM && S > 1;
+    Plan q;
+    q.block = T;
+    q.simdlen = S;
+    q.mode = S == 1 ? NEST_MODE_SPMD : d->mode;
+    q.reduce = d->reduce;
+    q.groups = T / S;
+    q.slot_bytes = sharing / q.groups;                  // split evenly
+    q.payload_bytes = payload;
+    q.fallback = smem_mode && payload > q.slot_bytes;
+    q.unroll = U;
+    q.smem_bytes = smem_mode ? sharing : 0;             // SPMD needs no sharing space
+    q.flags = d->flags;
+    q.outer = outer;
+    // one batch of U steps spans ceil(U/K) outer iterations of a group
+    const int64_t per_group = (U + K - 1) / K;
+    const int64_t denom = (int64_t)q.groups * per_group;
+    int64_t needed = (outer + denom - 1) / denom;
+    if (d->x_halo > 0) {
+        // x window (spmv_xwin.cuh): ring of 2^k >= 2R + 2H doubles, R = G*U rows per chunk,
+        // plus a double-buffered rowptr stage; always a persistent block schedule.
+        const int64_t R = (int64_t)q.groups * U;
+        const int64_t need = 2 * R + 2 * (int64_t)d->x_halo;
+        int32_t lg = 4;
+        while (((int64_t)1 << lg) < need) ++lg;
+        const int64_t bytes = ((int64_t)8 << lg) + 2 * (R + 1) * 8 + q.smem_bytes;
+        if (bytes > kMaxDynSmem)
+            return fail(NEST_ERR_UNSUPPORTED,
+                        "x_halo %d with %lld rows per chunk needs %lld B of shared memory (max %d)",
+                        d->x_halo, (long long)R, (long long)bytes, kMaxDynSmem);
+        q.x_halo = d->x_halo;
+        q.xw_log2 = lg;
+        q.smem_bytes = (int32_t)bytes;
+        if (d->num_teams > 0) {
+            q.grid = d->num_teams;
+        } else {
+            int64_t resident = 0;
+            nest_status s = resident_blocks(T, q.smem_bytes, &resident);
+            if (s != NEST_OK) return s;
+            q.grid = (int32_t)(needed < resident ? needed : resident);
+        }
+    } else if (d->num_teams > 0) {
+        q.grid = d->num_teams;
+    } else if ((d->flags & NEST_F_PERSISTENT_GRID) || q.fallback) {
+        int64_t resident = 0;
+        nest_status s = resident_blocks(T, q.smem_bytes, &resident);
+        if (s != NEST_OK) return s;
+        q.grid = (int32_t)(needed < resident ? needed : resident);
+    } else {
+        if (needed > INT32_MAX) needed = INT32_MAX;
+        q.grid = (int32_t)needed;
+    }
+    *p = q;
+    return NEST_OK;
+}
+
+nest_status make_plan(const nest_desc* d, int64_t outer, int32_t K, PayloadFn payload_of, Plan* p,
+                      bool spmv_window) {
+    int32_t T, sharing, U;
+    nest_status s = validate_desc(d, &T, &sharing, &U);
+    if (s != NEST_OK) return s;
+    return plan_core(d, outer, K, T, sharing, U, payload_of(U), p, spmv_window);
+}
+
+nest_status make_plan_fixed(const nest_desc* d, int64_t outer, int32_t K, int32_t payload, Plan* p,
+                            bool spmv_window) {
+    int32_t T, sharing, U;
+    nest_status s = validate_desc(d, &T, &sharing, &U);
+    if (s != NEST_OK) return s;
+    if (payload < 0) return fail(NEST_ERR_INVALID_ARG, "payload_bytes %d < 0", payload);
+    return plan_core(d, outer, K, T, sharing, U, payload, p, spmv_window);
+}
+
+// ------------------------------------------------ sharing-space fallback
+struct Scratch {
+    unsigned char* ptr = nullptr;
+    size_t bytes = 0;
+};
+static std::mutex g_scratch_mu;
+static Scratch g_scratch[64];
+
+nest_status fallback_scratch(size_t bytes, unsigned char** out) {
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
+    if (dev < 0 || dev >= 64) return fail(NEST_ERR_UNSUPPORTED, "device %d", dev);
+    std::lock_guard<std::mutex> lk(g_scratch_mu);
+    Scratch& s = g_scratch[dev];
+    if (s.bytes < bytes) {
+        if (s.ptr) {
+            e = cudaFree(s.ptr);   // synchronises: only on growth, never in steady state
+            s.ptr = nullptr;
+            s.bytes = 0;
+            if (e != cudaSuccess) return cuda_fail(e, "cudaFree(fallback)");
+        }
+        e = cudaMalloc(&s.ptr, bytes);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            return fail(NEST_ERR_NO_MEMORY, "fallback scratch of %zu bytes", bytes);
+        }
+        s.bytes = bytes;
+    }
+    *out = s.ptr;
+    return NEST_OK;
+}
+
+static nest_status prepare_fallback(const Plan& p, unsigned char** fb) {
+    *fb = nullptr;
+    if (!p.fallback) return NEST_OK;
+    const size_t bytes = (size_t)p.grid * (size_t)p.groups * (size_t)p.payload_bytes;
+    return fallback_scratch(bytes, fb);
+}
+
+// --------------------------------------------------------- device utilities
+__global__ void csr_validate_kernel(int64_t nrows, int64_t ncols, int64_t nnz,
+                                    const int64_t* __restrict__ rowptr,
+                                    const int32_t* __restrict__ col, int32_t* __restrict__ bad) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    const int64_t t0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t0 == 0 && (rowptr[0] != 0 || rowptr[nrows] != nnz)) atomicOr(bad, 1);
+    for (int64_t i = t0; i < nrows; i += stride)
+        if (rowptr[i + 1] < rowptr[i]) atomicOr(bad, 2);
+    for (int64_t k = t0; k < nnz; k += stride)
+        if (col[k] < 0 || (int64_t)col[k] >= ncols) atomicOr(bad, 4);
+}
+
+__global__ void l2_flush_kernel(uint4* __restrict__ buf, size_t n16, uint32_t salt) {
+    const size_t stride = (size_t)gridDim.x * blockDim.x;
+    for (size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < n16; i += stride)
+        buf[i] = make_uint4(salt, (uint32_t)i, salt ^ 0x9e3779b9u, (uint32_t)(i >> 32));
+}
+
+}  // namespace nest
+
+using namespace nest;
+
+static cudaStream_t as_stream(void* s) { return reinterpret_cast<cudaStream_t>(s); }
+
+NEST_API uint32_t nest_abi_version(void) { return NEST_ABI_VERSION; }
+
+NEST_API const char* nest_status_str(nest_status s) {
+    switch (s) {
+        case NEST_OK: return "NEST_OK";
+        case NEST_ERR_INVALID_ARG: return "NEST_ERR_INVALID_ARG";
+        case NEST_ERR_UNSUPPORTED: return "NEST_ERR_UNSUPPORTED";
+        case NEST_ERR_CUDA: return "NEST_ERR_CUDA";
+        case NEST_ERR_NCCL: return "NEST_ERR_NCCL";
+        case NEST_ERR_NO_MEMORY: return "NEST_ERR_NO_MEMORY";
+    }
+    return "NEST_ERR_UNKNOWN";
+}
+
+NEST_API const char* nest_last_error(void) { return nest::g_err; }
+
+NEST_API nest_status nest_plan(const nest_desc* desc, int64_t outer_iters, int32_t payload_bytes,
+                               nest_plan_info* out) {
+    if (!out) return fail(NEST_ERR_INVALID_ARG, "out is NULL");
+    Plan p;
+    nest_status s = make_plan_fixed(desc, outer_iters, 1, payload_bytes, &p, true);
+    if (s != NEST_OK) return s;
+    out->grid = p.grid;
+    out->block = p.block;
+    out->groups_per_team = p.groups;
+    out->slot_bytes = p.slot_bytes;
+    out->payload_bytes = p.payload_bytes;
+    out->uses_global_fallback = p.fallback;
+    out->outer_unroll = p.unroll;
+    out->smem_bytes = p.smem_bytes;
+    return NEST_OK;
+}
+
+NEST_API nest_status nest_spmv_csr_f64(const nest_desc* desc, int64_t nrows, int64_t ncols,
+                                       int64_t nnz, const int64_t* rowptr, const int32_t* colind,
+                                       const double* val, const double* x, double* y,
+                                       void* stream) {
+    if (nrows < 0 || ncols < 0 || nnz < 0)
+        return fail(NEST_ERR_INVALID_ARG, "negative extent (nrows %lld, ncols %lld, nnz %lld)",
+                    (long long)nrows, (long long)ncols, (long long)nnz);
+    if (ncols > INT32_MAX) return fail(NEST_ERR_INVALID_ARG, "ncols exceeds int32 column indices");
+    Plan p;
+    nest_status s = make_plan(desc, nrows, 1, spmv_payload, &p, true);
+    if (s != NEST_OK) return s;
+    if (nrows == 0) return NEST_OK;
+    if (!rowptr || !y) return fail(NEST_ERR_INVALID_ARG, "rowptr/y is NULL");
+    if (nnz > 0 && (!colind || !val || !x)) return fail(NEST_ERR_INVALID_ARG, "colind/val/x is NULL");
+    unsigned char* fb = nullptr;
+    if ((s = prepare_fallback(p, &fb)) != NEST_OK) return s;
+    if (p.x_halo > 0) return launch_spmv_xwin(p, nrows, ncols, rowptr, colind, val, x, y, fb, as_stream(stream));
+    return launch_spmv(p, (p.flags & NEST_F_STREAM_HINTS) != 0, nrows, rowptr, colind, val, x, y, fb,
+                       as_stream(stream));
+}
+
+static size_t align256(size_t b) { return (b + 255) & ~(size_t)255; }
+
+NEST_API size_t nest_spmv_hostio_workspace_bytes(int64_t nrows, int64_t ncols, int64_t nnz) {
+    if (nrows < 0 || ncols < 0 || nnz < 0) return 0;
+    return align256((size_t)(nrows + 1) * 8) + align256((size_t)nnz * 4) + align256((size_t)nnz * 8) +
+           align256((size_t)ncols * 8) + align256((size_t)nrows * 8);
+}
+
+NEST_API nest_status nest_spmv_csr_f64_hostio(const nest_desc* desc, int64_t nrows, int64_t ncols,
+                                              int64_t nnz, const int64_t* h_rowptr,
+                                              const int32_t* h_colind, const double* h_val,
+                                              const double* h_x, double* h_y, void* d_workspace,
+                                              size_t workspace_bytes, void* stream) {
+    if (nrows < 0 || ncols < 0 || nnz < 0) return fail(NEST_ERR_INVALID_ARG, "negative extent");
+    Plan p;
+    nest_status s = make_plan(desc, nrows, 1, spmv_payload, &p, true);
+    if (s != NEST_OK) return s;
+    if (nrows == 0) return NEST_OK;
+    const size_t need = nest_spmv_hostio_workspace_bytes(nrows, ncols, nnz);
+    if (!d_workspace || workspace_bytes < need)
+        return fail(NEST_ERR_INVALID_ARG, "workspace %zu bytes < %zu", workspace_bytes, need);
+    if (!h_rowptr || !h_y || (nnz > 0 && (!h_colind || !h_val || !h_x)))
+        return fail(NEST_ERR_INVALID_ARG, "host buffer is NULL");
+    unsigned char* w = static_cast<unsigned char*>(d_workspace);
+    int64_t* d_rowptr = reinterpret_cast<int64_t*>(w);
+    w += align256((size_t)(nrows + 1) * 8);
+    int32_t* d_col = reinterpret_cast<int32_t*>(w);
+    w += align256((size_t)nnz * 4);
+    double* d_val = reinterpret_cast<double*>(w);
+    w += align256((size_t)nnz * 8);
+    double* d_x = reinterpret_cast<double*>(w);
+    w += align256((size_t)ncols * 8);
+    double* d_y = reinterpret_cast<double*>(w);
+    unsigned char* fb = nullptr;
+    if ((s = prepare_fallback(p, &fb)) != NEST_OK) return s;
+    cudaStream_t st = as_stream(stream);
+    cudaError_t e;
+    if ((e = cudaMemcpyAsync(d_rowptr, h_rowptr, (size_t)(nrows + 1) * 8, cudaMemcpyHostToDevice, st)) ||
+        (nnz && (e = cudaMemcpyAsync(d_col, h_colind, (size_t)nnz * 4, cudaMemcpyHostToDevice, st))) ||
+        (nnz && (e = cudaMemcpyAsync(d_val, h_val, (size_t)nnz * 8, cudaMemcpyHostToDevice, st))) ||
+        (ncols && (e = cudaMemcpyAsync(d_x, h_x, (size_t)ncols * 8, cudaMemcpyHostToDevice, st))))
+        return cuda_fail(e, "host->device copy");
+    s = p.x_halo > 0 ? launch_spmv_xwin(p, nrows, ncols, d_rowptr, d_col, d_val, d_x, d_y, fb, st)
+                     : launch_spmv(p, (p.flags & NEST_F_STREAM_HINTS) != 0, nrows, d_rowptr, d_col, d_val,
+                                   d_x, d_y, fb, st);
+    if (s != NEST_OK) return s;
+    if ((e = cudaMemcpyAsync(h_y, d_y, (size_t)nrows * 8, cudaMemcpyDeviceToHost, st)))
+        return cuda_fail(e, "device->host copy");
+    return NEST_OK;
+}
+
+NEST_API nest_status nest_batched_matvec_f32(const nest_desc* desc, int64_t batch, int32_t m,
+                                             int32_t n, const float* A, const float* x, float* y,
+                                             void* stream) {
+    if (batch < 0 || m < 0 || n < 0) return fail(NEST_ERR_INVALID_ARG, "negative extent");
+    Plan p;
+    nest_status s = make_plan(desc, batch, m, batched_payload, &p);
+    if (s != NEST_OK) return s;
+    if (batch == 0 || m == 0) return NEST_OK;
+    if (!y || (n > 0 && (!A || !x))) return fail(NEST_ERR_INVALID_ARG, "A/x/y is NULL");
+    unsigned char* fb = nullptr;
+    if ((s = prepare_fallback(p, &fb)) != NEST_OK) return s;
+    return launch_batched(p, batch, m, n, A, x, y, fb, as_stream(stream));
+}
+
+NEST_API nest_status nest_nested_stencil_f64(const nest_desc* desc, int64_t nouter, int32_t L,
+                                             const double* in, const double* coef,
+                                             const double* w, double* out,
+                                             unsigned long long* visits, void* stream) {
+    if (nouter < 0 || L < 0) return fail(NEST_ERR_INVALID_ARG, "negative extent");
+    Plan p;
+    nest_status s = make_plan(desc, nouter, 1, stencil_payload, &p);
+    if (s != NEST_OK) return s;
+    if (nouter == 0) return NEST_OK;
+    if (!w || !out || (L > 0 && (!in || !coef))) return fail(NEST_ERR_INVALID_ARG, "in/coef/w/out is NULL");
+    unsigned char* fb = nullptr;
+    if ((s = prepare_fallback(p, &fb)) != NEST_OK) return s;
+    return launch_stencil(p, nouter, L, in, coef, w, out, visits, fb, as_stream(stream));
+}
+
+NEST_API nest_status nest_probe_mapping(const nest_desc* desc, int32_t* out_map, int64_t trip,
+                                        int32_t* hits, int32_t* owner, double* totals,
+                                        void* stream) {
+    if (!desc || desc->num_teams <= 0) return fail(NEST_ERR_INVALID_ARG, "probe needs num_teams > 0");
+    if (trip < 0) return fail(NEST_ERR_INVALID_ARG, "trip < 0");
+    if (!valid_simdlen(desc->simdlen)) return fail(NEST_ERR_INVALID_ARG, "simdlen %d", desc->simdlen);
+    const int32_t T = desc->threads_per_team ? desc->threads_per_team : kDefaultThreads;
+    const int64_t outer = (int64_t)desc->num_teams * (T / desc->simdlen);
+    Plan p;
+    nest_status s = make_plan(desc, outer, 1, probe_payload, &p);
+    if (s != NEST_OK) return s;
+    unsigned char* fb = nullptr;
+    if ((s = prepare_fallback(p, &fb)) != NEST_OK) return s;
+    return launch_probe(p, out_map, trip, hits, owner, totals, fb, as_stream(stream));
+}
+
+NEST_API nest_status nest_csr_validate(int64_t nrows, int64_t ncols, int64_t nnz,
+                                       const int64_t* rowptr, const int32_t* colind, int32_t* d_bad,
+                                       void* stream) {
+    if (nrows < 0 || ncols < 0 || nnz < 0 || !rowptr || !d_bad || (nnz > 0 && !colind))
+        return fail(NEST_ERR_INVALID_ARG, "bad arguments");
+    csr_validate_kernel<<<1184, 256, 0, as_stream(stream)>>>(nrows, ncols, nnz, rowptr, colind, d_bad);
+    const cudaError_t e = cudaGetLastError();
+    return e == cudaSuccess ? NEST_OK : cuda_fail(e, "csr_validate launch");
+}
+
+NEST_API nest_status nest_util_l2_flush(void* buf, size_t bytes, void* stream) {
+    if (!buf && bytes) return fail(NEST_ERR_INVALID_ARG, "buf is NULL");
+    static uint32_t salt = 1;
+    const size_t n16 = bytes / 16;
+    if (n16 == 0) return NEST_OK;
+    l2_flush_kernel<<<1184, 512, 0, as_stream(stream)>>>(static_cast<uint4*>(buf), n16, salt++);
+    const cudaError_t e = cudaGetLastError();
+    return e == cudaSuccess ? NEST_OK : cuda_fail(e, "l2_flush launch");
+}
+
+NEST_API nest_status nest_shutdown(void) {
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
+    std::lock_guard<std::mutex> lk(g_scratch_mu);
+    if (dev >= 0 && dev < 64 && g_scratch[dev].ptr) {
+        e = cudaFree(g_scratch[dev].ptr);
+        g_scratch[dev] = Scratch{};
+        if (e != cudaSuccess) return cuda_fail(e, "cudaFree(fallback)");
+    }
+    return NEST_OK;
+}

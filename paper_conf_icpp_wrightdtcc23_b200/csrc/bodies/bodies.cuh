@@ -1,0 +1,208 @@
+// bodies.cuh -- the fixed device loop bodies (a8, a9, a10, probe).
+//
+// Each body is the compile-time analogue of the outlined WorkFn plus the
+// sequential code of its parallel region (the loop body is
+// outlined into a function taking (iv, payload); the B200 build instantiates
+// it as a template instead of a function pointer -- the if-cascade of
+// PAPER.md:794-800 resolved at compile time).  Contract used by engine.cuh:
+//   Acc                         accumulator type of the simd reduction
+//   Loop {trip, ...}            loop state the SIMD main posts (generic payload)
+//   Step                        main-private state needed by the epilogue
+//   TeamShared                  per-team shared state (team_begin/team_end)
+//   steps(body)                 simd loops per outer iteration (K)
+//   prologue(i, r, st, fx, tsh) sequential code before simd loop r of outer
+//                               iteration i; side effects only if fx
+//   accum<OP>(L, j, acc)        WorkFn(j, args) folded into the accumulator
+//   epilogue(st, total)         sequential code after the loop (SIMD main)
+#pragma once
+
+#include <cstdint>
+
+#include "device/engine.cuh"
+
+namespace nest {
+
+// Streaming loads: L1 no-allocate + L2 evict-first policy (read once).
+__device__ __forceinline__ int32_t ld_stream(const int32_t* p) { return __ldcs(p); }
+__device__ __forceinline__ double ld_stream(const double* p) { return __ldcs(p); }
+
+// ---------------------------------------------------------------- a8 SpMV
+// sparse_matvec: outer loop over rows on "teams distribute
+// parallel for", inner loop over the row's nonzeros on "simd".  The product is
+// reduced in-group (R2) instead of the paper's atomic update.
+template <bool HINTS>
+struct SpmvBody {
+    using Acc = double;
+    struct Loop {
+        int64_t trip;   // nonzeros in the row (TripCount)
+        int64_t base;   // rowptr[i]
+    };
+    struct Step {
+        int64_t i;
+    };
+    static constexpr bool kTeamState = false;
+    struct TeamShared {
+        int unused;
+    };
+    const int64_t* rowptr;
+    const int32_t* col;
+    const double* val;
+    const double* x;
+    double* y;
+
+    static __device__ __forceinline__ int steps(const SpmvBody&) { return 1; }
+    static __device__ __forceinline__ void team_begin(TeamShared&) {}
+    static __device__ __forceinline__ void team_end(const SpmvBody&, TeamShared&) {}
+
+    __device__ __forceinline__ Loop prologue(int64_t i, int, Step& st, bool, TeamShared&) const {
+        st.i = i;
+        const int64_t b = __ldg(rowptr + i);
+        const int64_t e = __ldg(rowptr + i + 1);
+        return Loop{e - b, b};
+    }
+    template <int OP>
+    __device__ __forceinline__ double accum(const Loop& L, int64_t j, double acc) const {
+        const int64_t k = L.base + j;
+        const int32_t c = HINTS ? ld_stream(col + k) : __ldg(col + k);
+        const double v = HINTS ? ld_stream(val + k) : __ldg(val + k);
+        return Red<OP, double>::accum(acc, v, __ldg(x + c));
+    }
+    __device__ __forceinline__ void epilogue(const Step& st, double total) const { y[st.i] = total; }
+};
+
+// ------------------------------------------------------- a9 batched matvec
+// SU3_bench stand-in: outer loop over batches, a
+// sequential loop over the m rows inside the parallel region, a simd loop of
+// n iterations (the dot product) per row.
+struct BatchedBody {
+    using Acc = float;
+    struct Loop {
+        int64_t trip;    // n
+        int64_t base;    // (b*m + r)*n
+        int64_t xbase;   // b*n
+    };
+    struct Step {
+        int64_t out;     // b*m + r
+    };
+    static constexpr bool kTeamState = false;
+    struct TeamShared {
+        int unused;
+    };
+    const float* A;
+    const float* x;
+    float* y;
+    int32_t m, n;
+
+    static __device__ __forceinline__ int steps(const BatchedBody& b) { return b.m; }
+    static __device__ __forceinline__ void team_begin(TeamShared&) {}
+    static __device__ __forceinline__ void team_end(const BatchedBody&, TeamShared&) {}
+
+    __device__ __forceinline__ Loop prologue(int64_t b, int r, Step& st, bool, TeamShared&) const {
+        st.out = b * m + r;
+        return Loop{n, (b * m + r) * (int64_t)n, b * (int64_t)n};
+    }
+    template <int OP>
+    __device__ __forceinline__ float accum(const Loop& L, int64_t j, float acc) const {
+        return Red<OP, float>::accum(acc, __ldg(A + L.base + j), __ldg(x + L.xbase + j));
+    }
+    __device__ __forceinline__ void epilogue(const Step& st, float total) const { y[st.out] = total; }
+};
+
+// ---------------------------------------------- a10 nested stencil loop
+// "Benchmark kernel" stand-in with a data-dependent
+// sequential prologue and a non-idempotent side effect
+// that SPMD mode must guard: visits += 1.
+// The counter is aggregated per team in shared memory (one global atomic per
+// team); the count is still exactly one per outer iteration.
+struct StencilBody {
+    using Acc = double;
+    struct Loop {
+        int64_t trip;   // L, or 0 when w[i] == 0
+        int64_t base;   // 1 + i*L
+    };
+    struct Step {
+        int64_t i;
+        double scale;
+        int64_t skip;
+    };
+    static constexpr bool kTeamState = true;
+    struct TeamShared {
+        unsigned long long visits;
+    };
+    const double* in;
+    const double* coef;
+    const double* w;
+    double* out;
+    unsigned long long* visits;
+    int32_t L;
+
+    static __device__ __forceinline__ int steps(const StencilBody&) { return 1; }
+    static __device__ __forceinline__ void team_begin(TeamShared& t) {
+        if (threadIdx.x == 0) t.visits = 0ull;
+    }
+    static __device__ __forceinline__ void team_end(const StencilBody& b, TeamShared& t) {
+        if (threadIdx.x == 0 && b.visits && t.visits) atomicAdd(b.visits, t.visits);
+    }
+
+    __device__ __forceinline__ Loop prologue(int64_t i, int, Step& st, bool side_effects,
+                                             TeamShared& tsh) const {
+        const double scale = __ldg(w + i);
+        if (side_effects) atomicAdd_block(&tsh.visits, 1ull);
+        st.i = i;
+        st.scale = scale;
+        st.skip = (scale == 0.0);
+        return Loop{st.skip ? 0 : (int64_t)L, 1 + i * (int64_t)L};
+    }
+    template <int OP>
+    __device__ __forceinline__ double accum(const Loop& Lp, int64_t j, double acc) const {
+        const double* p = in + Lp.base + j;
+        const double t = (__ldg(p - 1) + 2.0 * __ldg(p)) + __ldg(p + 1);
+        return Red<OP, double>::accum(acc, __ldg(coef + j), t);
+    }
+    __device__ __forceinline__ void epilogue(const Step& st, double total) const {
+        out[st.i] = st.skip ? +0.0 : st.scale * total;
+    }
+};
+
+// ---------------------------------------------------------------- probe
+// One outer iteration per group; the simd loop body records coverage (hits),
+// the executing lane (owner, group 0 only) and counts iterations through the
+// reduction (totals[i] == trip under SUM).
+struct ProbeBody {
+    using Acc = double;
+    struct Loop {
+        int64_t trip;
+        int64_t base;   // the outer iteration (group) index
+    };
+    struct Step {
+        int64_t i;
+    };
+    static constexpr bool kTeamState = false;
+    struct TeamShared {
+        int unused;
+    };
+    int32_t* hits;
+    int32_t* owner;
+    double* totals;
+    int64_t trip;
+
+    static __device__ __forceinline__ int steps(const ProbeBody&) { return 1; }
+    static __device__ __forceinline__ void team_begin(TeamShared&) {}
+    static __device__ __forceinline__ void team_end(const ProbeBody&, TeamShared&) {}
+
+    __device__ __forceinline__ Loop prologue(int64_t i, int, Step& st, bool, TeamShared&) const {
+        st.i = i;
+        return Loop{trip, i};
+    }
+    template <int OP>
+    __device__ __forceinline__ double accum(const Loop& L, int64_t j, double acc) const {
+        if (hits) atomicAdd(hits + j, 1);
+        if (owner && L.base == 0) owner[j] = (int32_t)(threadIdx.x & 31u);
+        return Red<OP, double>::accum(acc, 1.0, 1.0);
+    }
+    __device__ __forceinline__ void epilogue(const Step& st, double total) const {
+        if (totals) totals[st.i] = total;
+    }
+};
+
+}  // namespace nest

@@ -1,0 +1,69 @@
+// dispatch.cuh -- host-side template dispatch from a runtime Plan to one
+// kernel instantiation nest_kernel<S, MODE, OP, U, Body>.  This is the B200
+// analogue of the paper's if-cascade over known outlined regions
+// (PAPER.md:794-800): every (simdlen, mode, reduction, unroll, body) is a
+// compile-time variant, so the hot loop has no indirect call.
+#pragma once
+
+#include "bodies/bodies.cuh"
+#include "internal.h"
+
+namespace nest {
+
+template <class Body, int U, int S, int MODE, int OP>
+nest_status launch_one(const Plan& p, const Body& body, unsigned char* fb, cudaStream_t st) {
+    nest_kernel<S, MODE, OP, U, Body><<<p.grid, p.block, p.smem_bytes, st>>>(body, p.outer,
+                                                                              p.slot_bytes, fb);
+    const cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "kernel launch");
+    return NEST_OK;
+}
+
+template <class Body, int U, int S, int MODE>
+nest_status dispatch_op(const Plan& p, const Body& b, unsigned char* fb, cudaStream_t st) {
+    switch (p.reduce) {
+        case RED_SUM: return launch_one<Body, U, S, MODE, RED_SUM>(p, b, fb, st);
+        case RED_MAX: return launch_one<Body, U, S, MODE, RED_MAX>(p, b, fb, st);
+        case RED_MIN: return launch_one<Body, U, S, MODE, RED_MIN>(p, b, fb, st);
+    }
+    return fail(NEST_ERR_INVALID_ARG, "reduce %d", p.reduce);
+}
+
+template <class Body, int U, int S>
+nest_status dispatch_mode(const Plan& p, const Body& b, unsigned char* fb, cudaStream_t st) {
+    if constexpr (S == 1) {
+        return dispatch_op<Body, U, 1, MODE_SPMD>(p, b, fb, st);
+    } else {
+        switch (p.mode) {
+            case MODE_SPMD: return dispatch_op<Body, U, S, MODE_SPMD>(p, b, fb, st);
+            case MODE_GENERIC_SMEM: return dispatch_op<Body, U, S, MODE_GENERIC_SMEM>(p, b, fb, st);
+            case MODE_GENERIC_SHFL: return dispatch_op<Body, U, S, MODE_GENERIC_SHFL>(p, b, fb, st);
+        }
+    }
+    return fail(NEST_ERR_INVALID_ARG, "mode %d", p.mode);
+}
+
+template <class Body, int U>
+nest_status dispatch_simdlen(const Plan& p, const Body& b, unsigned char* fb, cudaStream_t st) {
+    switch (p.simdlen) {
+        case 1: return dispatch_mode<Body, U, 1>(p, b, fb, st);
+        case 2: return dispatch_mode<Body, U, 2>(p, b, fb, st);
+        case 4: return dispatch_mode<Body, U, 4>(p, b, fb, st);
+        case 8: return dispatch_mode<Body, U, 8>(p, b, fb, st);
+        case 16: return dispatch_mode<Body, U, 16>(p, b, fb, st);
+        case 32: return dispatch_mode<Body, U, 32>(p, b, fb, st);
+    }
+    return fail(NEST_ERR_INVALID_ARG, "simdlen %d", p.simdlen);
+}
+
+template <class Body>
+nest_status dispatch(const Plan& p, const Body& b, unsigned char* fb, cudaStream_t st) {
+    switch (p.unroll) {
+        case 1: return dispatch_simdlen<Body, 1>(p, b, fb, st);
+        case 2: return dispatch_simdlen<Body, 2>(p, b, fb, st);
+        case 4: return dispatch_simdlen<Body, 4>(p, b, fb, st);
+    }
+    return fail(NEST_ERR_INVALID_ARG, "outer_unroll %d", p.unroll);
+}
+
+}  // namespace nest

@@ -1,0 +1,73 @@
+// internal.h -- host-side declarations shared by the translation units of
+// libnest.so (never exported; the ABI is include/nest.h).
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "nest.h"
+
+#define NEST_API extern "C" __attribute__((visibility("default")))
+
+namespace nest {
+
+// a1: the resolved launch plan.
+struct Plan {
+    int32_t grid = 0;
+    int32_t block = 0;
+    int32_t simdlen = 0;
+    int32_t mode = 0;      // effective mode (S == 1 runs SPMD: PAPER.md:691-693)
+    int32_t reduce = 0;
+    int32_t groups = 0;    // G
+    int32_t slot_bytes = 0;
+    int32_t payload_bytes = 0;
+    int32_t fallback = 0;
+    int32_t unroll = 1;    // U
+    int32_t smem_bytes = 0;
+    uint32_t flags = 0;
+    int64_t outer = 0;
+    int32_t x_halo = 0;    // SpMV x window half-width (0 = none)
+    int32_t xw_log2 = 0;   // ring of 2^xw_log2 doubles
+};
+
+// Record a thread-local error message and return `s`.
+nest_status fail(nest_status s, const char* fmt, ...) __attribute__((format(printf, 2, 3)));
+nest_status cuda_fail(cudaError_t e, const char* what);
+
+// Validate `d` and compute the plan for `outer` outer iterations of a body
+// with `steps_per_outer` simd loops each; payload_of(U) is the generic payload
+// one group posts per simd batch at unroll U.
+using PayloadFn = int32_t (*)(int32_t unroll);
+nest_status make_plan(const nest_desc* d, int64_t outer, int32_t steps_per_outer,
+                      PayloadFn payload_of, Plan* p, bool spmv_window = false);
+// as make_plan with a fixed payload (the nest_plan ABI entry)
+nest_status make_plan_fixed(const nest_desc* d, int64_t outer, int32_t steps_per_outer,
+                            int32_t payload_bytes, Plan* p, bool spmv_window = false);
+
+// Library-owned global fallback for the sharing space:
+// grown lazily, never shrunk, released by nest_shutdown().
+nest_status fallback_scratch(size_t bytes, unsigned char** out);
+
+// Payload bytes a body posts per simd batch for a given unroll.
+int32_t spmv_payload(int32_t U);
+int32_t batched_payload(int32_t U);
+int32_t stencil_payload(int32_t U);
+int32_t probe_payload(int32_t U);
+
+// Kernel launchers (one translation unit per body).
+nest_status launch_spmv(const Plan& p, bool hints, int64_t nrows, const int64_t* rowptr,
+                        const int32_t* col, const double* val, const double* x, double* y,
+                        unsigned char* fb, cudaStream_t st);
+nest_status launch_spmv_xwin(const Plan& p, int64_t nrows, int64_t ncols, const int64_t* rowptr,
+                             const int32_t* col, const double* val, const double* x, double* y,
+                             unsigned char* fb, cudaStream_t st);
+nest_status launch_batched(const Plan& p, int64_t batch, int32_t m, int32_t n, const float* A,
+                           const float* x, float* y, unsigned char* fb, cudaStream_t st);
+nest_status launch_stencil(const Plan& p, int64_t nouter, int32_t L, const double* in,
+                           const double* coef, const double* w, double* out,
+                           unsigned long long* visits, unsigned char* fb, cudaStream_t st);
+nest_status launch_probe(const Plan& p, int32_t* out_map, int64_t trip, int32_t* hits,
+                         int32_t* owner, double* totals, unsigned char* fb, cudaStream_t st);
+
+}  // namespace nest

@@ -1,0 +1,76 @@
+"""a12: row-partitioned multi-GPU SpMV, one process per GPU (north_star; the
+paper itself is single-GPU).
+
+torch.distributed is the plumbing: it broadcasts the 128-byte NCCL unique id
+that libnest.so's communicator is built from.  The all-gather of x and the
+local SpMV run inside libnest.so (``nest_spmv_csr_f64_dist``), on the caller's
+stream.
+"""
+from __future__ import annotations
+
+import ctypes
+
+from . import _nest as N
+from .api import _dev, _stream, _torch, check, make_desc
+
+
+def shard_rows(n: int, nranks: int, rank: int):
+    """Equal-row partition: chunk = ceil(n/P); rank r owns
+    [r*chunk, min((r+1)*chunk, n)).  Returns (chunk, row_begin, nrows_local)."""
+    if nranks <= 0 or not 0 <= rank < nranks or n < 0:
+        raise ValueError("bad partition arguments")
+    chunk = -(-n // nranks)
+    b = min(rank * chunk, n)
+    return chunk, b, min(b + chunk, n) - b
+
+
+class Comm:
+    """A libnest-owned NCCL communicator over the ranks of a torch process group."""
+
+    def __init__(self, group=None):
+        torch = _torch()
+        import torch.distributed as dist
+        self.rank = dist.get_rank(group)
+        self.nranks = dist.get_world_size(group)
+        uid = (ctypes.c_uint8 * 128)()
+        if self.rank == 0:
+            check(N.nest_comm_unique_id(uid), "nest_comm_unique_id")
+        obj = [bytes(uid)]
+        dist.broadcast_object_list(obj, src=0, group=group)
+        uid = (ctypes.c_uint8 * 128).from_buffer_copy(obj[0])
+        self._h = ctypes.c_void_p()
+        check(N.nest_comm_init(uid, self.nranks, self.rank, ctypes.byref(self._h)), "nest_comm_init")
+        self._torch = torch
+
+    def close(self):
+        if self._h:
+            check(N.nest_comm_destroy(self._h), "nest_comm_destroy")
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def spmv_csr_f64(self, nrows_global, ncols_global, rowptr, colind, val, x_local, x_full,
+                     y_local=None, *, stream=None, **cfg):
+        """y_local = A[local rows] @ x after all-gathering x (x_full is scratch/output)."""
+        torch = self._torch
+        nrows_local = rowptr.numel() - 1
+        nnz = val.numel()
+        xchunk = -(-ncols_global // self.nranks)
+        if y_local is None:
+            y_local = torch.empty(nrows_local, dtype=torch.float64, device=val.device)
+        d = make_desc(**cfg)
+        check(N.nest_spmv_csr_f64_dist(ctypes.byref(d), self._h, nrows_global, ncols_global,
+                                       nrows_local, nnz,
+                                       _dev(rowptr, torch.int64, nrows_local + 1, "rowptr"),
+                                       _dev(colind, torch.int32, nnz, "colind"),
+                                       _dev(val, torch.float64, nnz, "val"),
+                                       _dev(x_local, torch.float64, xchunk, "x_local"),
+                                       _dev(x_full, torch.float64, xchunk * self.nranks, "x_full"),
+                                       _dev(y_local, torch.float64, nrows_local, "y_local"),
+                                       _stream(stream)),
+              "nest_spmv_csr_f64_dist")
+        return y_local

@@ -1,0 +1,35 @@
+"""Run one SpMV variant a few times (for ncu captures).  Usage:
+python scripts/one_spmv.py --spec CFG2 --S 8 --mode spmd --U 1 --hints 0 --iters 3"""
+import argparse
+import os
+import sys
+
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import paper_conf_icpp_wrightdtcc23_b200 as P  # noqa: E402
+from nestgen import recipes as R  # noqa: E402
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--spec", default="CFG2")
+ap.add_argument("--S", type=int, default=8)
+ap.add_argument("--mode", default="spmd")
+ap.add_argument("--U", type=int, default=1)
+ap.add_argument("--T", type=int, default=256)
+ap.add_argument("--hints", type=int, default=0)
+ap.add_argument("--persistent", type=int, default=0)
+ap.add_argument("--iters", type=int, default=3)
+ap.add_argument("--halo", type=int, default=0)
+a = ap.parse_args()
+spec = getattr(R, a.spec)
+rp, col, val = R.spmv_matrix(spec)
+x = R.spmv_x(spec)
+t = [torch.from_numpy(v).cuda() for v in (rp, col, val, x)]
+y = torch.empty(spec.nrows, dtype=torch.float64, device="cuda")
+flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
+for _ in range(a.iters):
+    P.l2_flush(flush)
+    P.spmv_csr_f64(*t, y, simdlen=a.S, mode=a.mode, outer_unroll=a.U, stream_hints=bool(a.hints),
+                   threads_per_team=a.T, persistent=bool(a.persistent), x_halo=a.halo)
+torch.cuda.synchronize()
+print("done")

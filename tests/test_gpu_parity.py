@@ -1,0 +1,343 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle on the
+same seeded inputs.  Bars (north_star; R3/R4):
+  * integer and index outputs, integer-valued fp reductions: bit-exact;
+  * general fp: |gpu - oracle| <= tol * abs_ref per row, tol = 1e-12 (fp64),
+    1e-5 (fp32), abs_ref = sum |terms| (cancellation-safe); abs_ref == 0
+    requires an exact +0.0;
+  * MAX/MIN: equal by value (the sign of a zero tie is unordered);
+  * the modes (SPMD, GENERIC_SMEM, GENERIC_SHFL) and U agree bit-for-bit at
+    the same simdlen.
+"""
+import numpy as np
+import pytest
+
+import oracle
+from nestgen import recipes as R
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+SIMDLENS = (1, 2, 4, 8, 16, 32)
+MODES = ("spmd", "generic_smem", "generic_shfl")
+
+
+@pytest.fixture(scope="module")
+def P():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_icpp_wrightdtcc23_b200 as P
+    return P
+
+
+def dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+def host(t):
+    return t.cpu().numpy()
+
+
+def assert_close(y, ref, absref, tol):
+    y = np.asarray(y, np.float64)
+    zero = absref == 0
+    assert np.all(y[zero] == 0.0) and not np.signbit(y[zero]).any(), "abs_ref == 0 must give +0.0"
+    err = np.abs(y - ref)
+    bad = err > tol * absref
+    assert not bad.any(), f"{bad.sum()} rows beyond {tol}*abs: worst {np.max(err[~zero] / absref[~zero]):.3e}"
+
+
+def bits(a):
+    a = np.ascontiguousarray(a)
+    return a.view(np.int64 if a.dtype == np.float64 else np.int32)
+
+
+# ------------------------------------------------------------------ a2/a5/a6 probe
+@pytest.mark.parametrize("S", SIMDLENS)
+@pytest.mark.parametrize("mode", MODES)
+@pytest.mark.parametrize("T", [32, 256, 1024])
+def test_probe_mapping(P, S, mode, T):
+    teams = 3
+    G = T // S
+    for trip in sorted({0, 1, max(S - 1, 0), S, S + 1, 3 * S + 1, 77}):
+        mp, hits, owner, totals = P.probe_mapping(teams, trip, simdlen=S, mode=mode, threads_per_team=T)
+        ref = oracle.group_map(T, S)
+        m = host(mp).reshape(teams, T, 5)
+        for b in range(teams):
+            assert np.array_equal(m[b], ref)
+        assert np.all(host(hits) == teams * G)                       # every j once per group
+        assert np.array_equal(host(owner), oracle.simd_owner(trip, S))  # Fig 8 owner
+        assert np.all(host(totals) == float(trip))                   # reduction of the counts
+
+
+def test_probe_generic_fallback(P):
+    # 0-byte slots force the global fallback of the sharing space
+    for S in (2, 4, 32):
+        for sharing in (64, 2048, 16):
+            _, hits, owner, totals = P.probe_mapping(5, 40, simdlen=S, mode="generic_smem",
+                                                     sharing_bytes=sharing)
+            assert np.all(host(hits) == 5 * 256 // S)
+            assert np.array_equal(host(owner), oracle.simd_owner(40, S))
+            assert np.all(host(totals) == 40.0)
+
+
+# ------------------------------------------------------------------ a8 SpMV
+@pytest.fixture(scope="module")
+def cfg1():
+    out = {}
+    for spec in (R.CFG1, R.CFG1.integer()):
+        rp, col, val, x = R.spmv_inputs(spec)
+        y, a = oracle.spmv_csr_f64(rp, col, val, x)
+        out[spec.values] = (rp, col, val, x, y, a)
+    return out
+
+
+@pytest.mark.parametrize("S", SIMDLENS)
+@pytest.mark.parametrize("U", [1, 2, 4])
+def test_spmv_cfg1_all_modes(P, cfg1, S, U):
+    for values in ("int", "real"):
+        rp, col, val, x, yref, aref = cfg1[values]
+        t = [dev(rp), dev(col), dev(val), dev(x)]
+        ys = {}
+        for mode in MODES:
+            for hints in (False, True):
+                y = host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, outer_unroll=U, stream_hints=hints))
+                ys[(mode, hints)] = y
+                if values == "int":
+                    assert np.array_equal(bits(y), bits(yref)), (mode, hints)
+                else:
+                    assert_close(y, yref, aref, 1e-12)
+        first = next(iter(ys.values()))
+        for k, y in ys.items():
+            assert np.array_equal(bits(y), bits(first)), f"mode/hints {k} differs bitwise"
+
+
+def test_spmv_unroll_and_simdlen_integer_invariance(P, cfg1):
+    rp, col, val, x, yref, _ = cfg1["int"]
+    t = [dev(rp), dev(col), dev(val), dev(x)]
+    for S in SIMDLENS:
+        for T in (32, 128, 512, 1024):
+            for teams in (0, 1, 3):
+                y = host(P.spmv_csr_f64(*t, simdlen=S, threads_per_team=T, num_teams=teams))
+                assert np.array_equal(bits(y), bits(yref)), (S, T, teams)
+
+
+@pytest.mark.parametrize("op", ["max", "min"])
+def test_spmv_max_min(P, cfg1, op):
+    rp, col, val, x, _, _ = cfg1["real"]
+    yref, _ = oracle.spmv_csr_f64(rp, col, val, x, op=op)
+    t = [dev(rp), dev(col), dev(val), dev(x)]
+    for S in SIMDLENS:
+        for mode in MODES:
+            y = host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, reduce=op))
+            assert np.array_equal(y, yref), (S, mode)
+
+
+def _rows_matrix(lens, ncols, seed):
+    rng = np.random.default_rng(seed)
+    rp = np.concatenate([[0], np.cumsum(lens)]).astype(np.int64)
+    col = np.concatenate([np.sort(rng.choice(ncols, L, replace=False)) for L in lens] or [[]]).astype(np.int32)
+    val = rng.integers(-4, 5, rp[-1]).astype(np.float64)
+    x = rng.integers(-8, 9, ncols).astype(np.float64)
+    return rp, col, val, x
+
+
+def test_spmv_edge_rows(P):
+    # empty rows, a lone row, tails for every S (33, 64 nnz), a long row, ragged count
+    lens = [0, 0, 1, 33, 64, 0, 1000, 7, 31, 32, 5] * 7 + [2]
+    rp, col, val, x = _rows_matrix(lens, 2000, 3)
+    yref, _ = oracle.spmv_csr_f64(rp, col, val, x)
+    t = [dev(rp), dev(col), dev(val), dev(x)]
+    for S in SIMDLENS:
+        for mode in MODES:
+            for U in (1, 2, 4):
+                for sharing in (0, 64):
+                    y = host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, outer_unroll=U, sharing_bytes=sharing))
+                    assert np.array_equal(bits(y), bits(yref)), (S, mode, U, sharing)
+    # empty rows give +0.0 and MAX gives -inf
+    y = host(P.spmv_csr_f64(*t, simdlen=8, reduce="max"))
+    assert y[0] == -np.inf
+
+
+def test_spmv_zero_nnz_and_zero_rows(P):
+    rp = np.zeros(6, np.int64)
+    y = host(P.spmv_csr_f64(dev(rp), torch.zeros(0, dtype=torch.int32, device="cuda"),
+                            torch.zeros(0, dtype=torch.float64, device="cuda"),
+                            torch.zeros(3, dtype=torch.float64, device="cuda"), simdlen=4, mode="generic_smem"))
+    assert np.all(y == 0) and not np.signbit(y).any()
+    y0 = P.spmv_csr_f64(torch.zeros(1, dtype=torch.int64, device="cuda"),
+                        torch.zeros(0, dtype=torch.int32, device="cuda"),
+                        torch.zeros(0, dtype=torch.float64, device="cuda"),
+                        torch.zeros(3, dtype=torch.float64, device="cuda"))
+    assert y0.numel() == 0
+
+
+def test_csr_validate(P, cfg1):
+    rp, col, val, x, _, _ = cfg1["real"]
+    assert P.csr_validate(dev(rp), dev(col), 1024) == 0
+    bad = col.copy()
+    bad[5] = 1024
+    assert P.csr_validate(dev(rp), dev(bad), 1024) & 4
+    rp2 = rp.copy()
+    rp2[10] = rp2[12]
+    assert P.csr_validate(dev(rp2), dev(col), 1024) & 2
+
+
+def test_spmv_hostio_e2e(P, cfg1):
+    rp, col, val, x, yref, aref = cfg1["real"]
+    pin = lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory()
+    hy = torch.empty(rp.size - 1, dtype=torch.float64).pin_memory()
+    ws = torch.empty(P.hostio_workspace_bytes(rp.size - 1, x.size, val.size), dtype=torch.uint8, device="cuda")
+    P.spmv_csr_f64_hostio(pin(rp), pin(col), pin(val), pin(x), hy, ws, simdlen=8)
+    torch.cuda.synchronize()
+    assert_close(hy.numpy(), yref, aref, 1e-12)
+
+
+def test_spmv_cfg2_full_size_sampled(P):
+    """BASELINE configs[1] at full size (10M rows) in the bench launch
+    configurations; sampled rows compared against the oracle run on the same
+    rows regenerated independently."""
+    spec = R.CFG2
+    rp, col, val = R.spmv_matrix(spec)
+    x = R.spmv_x(spec)
+    t = [dev(rp), dev(col), dev(val), dev(x)]
+    rng = np.random.default_rng(7)
+    starts = np.concatenate([[0, spec.nrows - 64], rng.integers(0, spec.nrows - 64, 30)])
+    ref = {}
+    for s in starts:
+        rpl, cl, vl = R.spmv_matrix(spec, row_begin=int(s), nrows=64)
+        ref[int(s)] = oracle.spmv_csr_f64(rpl, cl, vl, x)
+    for S in SIMDLENS:
+        for mode in MODES:
+            for U, hints in ((1, False), (2, True), (4, True)):
+                y = host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, outer_unroll=U, stream_hints=hints))
+                for s, (yr, ar) in ref.items():
+                    assert_close(y[s:s + 64], yr, ar, 1e-12)
+    del t
+    torch.cuda.empty_cache()
+
+
+# ------------------------------------------------------------------ a9 batched
+@pytest.fixture(scope="module")
+def batched():
+    out = {}
+    B = 777
+    for values in ("int", "real"):
+        A, x = R.batched_inputs(B, values=values)
+        y, a = oracle.batched_matvec_f32(A, x, B)
+        out[values] = (B, A, x, y, a)
+    return out
+
+
+@pytest.mark.parametrize("S", SIMDLENS)
+@pytest.mark.parametrize("mode", MODES)
+def test_batched(P, batched, S, mode):
+    ys = []
+    for values in ("int", "real"):
+        B, A, x, yref, aref = batched[values]
+        for U in (1, 2, 4):
+            y = host(P.batched_matvec_f32(dev(A), dev(x), B, simdlen=S, mode=mode, outer_unroll=U))
+            if values == "int":
+                assert np.array_equal(bits(y), bits(yref))
+            else:
+                assert_close(y, yref, aref, 1e-5)
+                ys.append(y)
+    assert all(np.array_equal(bits(ys[0]), bits(v)) for v in ys)
+
+
+@pytest.mark.parametrize("op", ["max", "min"])
+def test_batched_max_min_and_rect(P, op):
+    B, m, n = 300, 5, 37
+    A, x = R.batched_inputs(B, m, n)
+    yref, _ = oracle.batched_matvec_f32(A, x, B, m, n, op=op)
+    for S in (1, 4, 32):
+        y = host(P.batched_matvec_f32(dev(A), dev(x), B, m, n, simdlen=S, reduce=op, mode="generic_smem"))
+        assert np.array_equal(y, yref)
+
+
+# ------------------------------------------------------------------ a10 stencil
+@pytest.mark.parametrize("L", R.STENCIL_LS + (1, 33))
+@pytest.mark.parametrize("mode", MODES)
+def test_stencil(P, L, mode):
+    N = 4099
+    for values in ("int", "real"):
+        inp, coef, w = R.stencil_inputs(N, L, values=values)
+        yref, aref, vref = oracle.nested_stencil_f64(inp, coef, w, N, L)
+        t = [dev(inp), dev(coef), dev(w)]
+        outs = []
+        for S in SIMDLENS:
+            for U in (1, 2):
+                visits = torch.zeros(1, dtype=torch.int64, device="cuda")
+                y = host(P.nested_stencil_f64(*t, N, L, visits=visits, simdlen=S, mode=mode, outer_unroll=U))
+                assert int(visits.item()) == vref == N            # guarded side effect: once per i
+                if values == "int":
+                    assert np.array_equal(bits(y), bits(yref)), (S, U)
+                else:
+                    assert_close(y, yref, aref, 1e-12)
+                outs.append(y)
+
+
+def test_stencil_max_and_cfg3_full(P):
+    N = 1 << 20
+    for L in (4, 64):
+        inp, coef, w = R.stencil_inputs(N, L)
+        yref, aref, _ = oracle.nested_stencil_f64(inp, coef, w, N, L)
+        t = [dev(inp), dev(coef), dev(w)]
+        for S in (1, 8, 32):
+            for mode in MODES:
+                y = host(P.nested_stencil_f64(*t, N, L, simdlen=S, mode=mode))
+                assert_close(y, yref, aref, 1e-12)
+        ymax, _, _ = oracle.nested_stencil_f64(inp, coef, w, N, L, op="max")
+        assert np.array_equal(host(P.nested_stencil_f64(*t, N, L, simdlen=16, reduce="max")), ymax)
+
+
+# ------------------------------------------------------------------ a8 SpMV, x window
+@pytest.fixture(scope="module")
+def banded():
+    out = {}
+    for values in ("int", "real"):
+        spec = R.SpmvSpec("band", 4242, 50_000, 50_000, 0, 20, band_w=700, far_den=8, values=values)
+        rp, col, val, x = R.spmv_inputs(spec)
+        y, a = oracle.spmv_csr_f64(rp, col, val, x)
+        out[values] = (rp, col, val, x, y, a)
+    return out
+
+
+@pytest.mark.parametrize("S", SIMDLENS)
+@pytest.mark.parametrize("mode", MODES)
+def test_spmv_xwin(P, banded, S, mode):
+    for values in ("int", "real"):
+        rp, col, val, x, yref, aref = banded[values]
+        t = [dev(rp), dev(col), dev(val), dev(x)]
+        for halo, U, T, teams in ((700, 1, 256, 0), (64, 2, 512, 0), (4096, 4, 256, 0),
+                                  (1, 1, 1024, 0), (700, 2, 256, 5), (3000, 1, 128, 1)):
+            y = host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, outer_unroll=U, threads_per_team=T,
+                                    x_halo=halo, num_teams=teams))
+            if values == "int":
+                assert np.array_equal(bits(y), bits(yref)), (halo, U, T, teams)
+            else:
+                assert_close(y, yref, aref, 1e-12)
+
+
+def test_spmv_xwin_cfg1_and_rectangular(P, cfg1):
+    rp, col, val, x, yref, aref = cfg1["int"]
+    t = [dev(rp), dev(col), dev(val), dev(x)]
+    for S in (1, 8, 32):
+        for halo in (1, 100, 5000):
+            y = host(P.spmv_csr_f64(*t, simdlen=S, x_halo=halo, mode="generic_smem", sharing_bytes=64))
+            assert np.array_equal(bits(y), bits(yref))
+    # more rows than columns: windows past the last column are empty
+    rows = [[(c, 1.0) for c in (0, 3)]] * 3000
+    rp2 = np.arange(0, 2 * 3000 + 1, 2, dtype=np.int64)
+    col2 = np.tile(np.array([0, 3], np.int32), 3000)
+    x2 = np.array([1.5, 0, 0, 2.0])
+    y = host(P.spmv_csr_f64(dev(rp2), dev(col2), dev(np.ones(6000)), dev(x2), simdlen=2, x_halo=8))
+    assert np.all(y == 3.5)
+    del rows
+
+
+def test_spmv_xwin_too_big_is_unsupported(P, cfg1):
+    rp, col, val, x, _, _ = cfg1["int"]
+    with pytest.raises(P.NestError) as e:
+        P.spmv_csr_f64(dev(rp), dev(col), dev(val), dev(x), simdlen=1, threads_per_team=1024,
+                       outer_unroll=4, x_halo=20000)
+    assert e.value.status == 2
