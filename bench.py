@@ -1,0 +1,385 @@
+"""Benchmark: the three-level CSR SpMV hot path on B200 (BASELINE.json metric
+"3-level SpMV GB/s vs HBM peak; speedup over simd-folded 2-level mapping").
+
+One step = one y = A x over BASELINE.json configs[1] (10M x 10M CSR, nnz/row
+U{4..12} banded+far, fp64) through the C ABI, in the best (simdlen, mode,
+variant) found by a short untimed autotune; the simd-folded two-level mapping
+(simdlen = 1) is timed the same way for the speedup.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+
+N > 1 (torchrun, one rank per GPU): the row-partitioned SpMV with the NCCL
+all-gather of x (BASELINE.json configs[4] scheme), weak scaling with 10M rows
+per rank.  --impl reference times the CPU oracle (the only reference this
+paper-only tier has) on the same workload.  Prints ONE JSON line on rank 0.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+from nestgen import recipes as R  # noqa: E402
+
+METRIC = "3-level SpMV GB/s vs HBM peak; speedup over simd-folded 2-level mapping"
+UNIT = "GB/s"
+SPEC = R.CFG2
+
+
+def alg_bytes(nrows: int, ncols: int, nnz: int) -> int:
+    """Algorithmic bytes of one SpMV: the CSR arrays once,
+    x once, y written once."""
+    return nnz * (8 + 4) + (nrows + 1) * 8 + nrows * 8 + ncols * 8
+
+
+def peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            p = json.load(f)
+        return float(p["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md)"
+
+
+class ClockSampler:
+    """nvidia-smi-equivalent clock / throttle sampling through NVML, run during
+    the timed region."""
+
+    def __init__(self, index: int, period: float = 0.002):
+        self.samples, self.reasons = [], set()
+        self.max_mhz = None
+        self._stop = threading.Event()
+        self._period = period
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self._nv = pynvml
+            self._h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self._h, pynvml.NVML_CLOCK_SM)
+        except Exception:
+            self._nv = None
+        self._t = threading.Thread(target=self._run, daemon=True)
+
+    def _run(self):
+        nv = self._nv
+        names = {}
+        if nv is not None:
+            for k in ("HwSlowdown", "HwThermalSlowdown", "SwThermalSlowdown", "SwPowerCap",
+                      "HwPowerBrakeSlowdown", "SyncBoost", "ApplicationsClocksSetting", "GpuIdle"):
+                v = getattr(nv, "nvmlClocksEventReason" + k, None) or getattr(nv, "nvmlClocksThrottleReason" + k, None)
+                if v is not None:
+                    names[k] = v
+        while not self._stop.is_set():
+            if nv is not None:
+                try:
+                    self.samples.append(nv.nvmlDeviceGetClockInfo(self._h, nv.NVML_CLOCK_SM))
+                    r = nv.nvmlDeviceGetCurrentClocksEventReasons(self._h)
+                    for k, bit in names.items():
+                        if r & bit and k != "GpuIdle":
+                            self.reasons.add(k)
+                except Exception:
+                    pass
+            time.sleep(self._period)
+
+    def __enter__(self):
+        self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        self._t.join()
+
+    def summary(self):
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
+                "sm_max_mhz": self.max_mhz, "samples": len(self.samples),
+                "reasons": sorted(self.reasons)}
+
+
+# ---------------------------------------------------------------- CPU oracle
+def cpu_baseline(spec, min_seconds=10.0, max_seconds=30.0):
+    """The oracle as it stands (plain sequential C, 1 thread) on a bounded
+    sample: whole passes of the same matrix until >= min_seconds."""
+    import oracle
+    rp, col, val = R.spmv_matrix(spec)
+    x = R.spmv_x(spec)
+    B = alg_bytes(spec.nrows, spec.ncols, val.size)
+    passes, t_total = 0, 0.0
+    while t_total < min_seconds and (passes == 0 or t_total + t_total / passes < max_seconds):
+        t0 = time.perf_counter()
+        oracle.spmv_csr_f64(rp, col, val, x)
+        t_total += time.perf_counter() - t0
+        passes += 1
+    return {"value": B * passes / t_total / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"{passes} full passes of {spec.name} ({spec.nrows} rows, {val.size} nnz), "
+                      f"{t_total:.1f} s single-threaded C (oracle/oracle.c)"}
+
+
+def run_reference(args, rank, world):
+    """--impl reference: the oracle on the box's host cores, rank 0 only."""
+    if rank != 0:
+        return
+    import oracle
+    spec = SPEC
+    rp, col, val = R.spmv_matrix(spec)
+    x = R.spmv_x(spec)
+    B = alg_bytes(spec.nrows, spec.ncols, val.size)
+    for _ in range(args.warmup):
+        oracle.spmv_csr_f64(rp, col, val, x)
+    ts = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        oracle.spmv_csr_f64(rp, col, val, x)
+        ts.append(time.perf_counter() - t0)
+    ms = 1e3 * sum(ts) / len(ts)
+    value = B / (ms / 1e3) / 1e9
+    line = {"metric": METRIC, "value": value, "unit": UNIT, "impl": "reference", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": f"{spec.name}: CSR SpMV fp64 {spec.nrows}x{spec.ncols}, nnz/row "
+                                   f"U{{{spec.nnz_min}..{spec.nnz_max}}} banded+far (W={spec.band_w}, "
+                                   f"far 1/{spec.far_den})", "nnz": int(val.size), "alg_bytes": B},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
+                             "sample": f"the full {spec.name} matrix per step, single-threaded C oracle"},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ---------------------------------------------------------------- GPU arm
+CANDIDATES = [
+    # (simdlen, mode, outer_unroll, threads, x_halo, stream_hints)
+    (1, "spmd", 1, 256, 0, False),
+    (1, "spmd", 2, 256, 0, False),
+    (2, "spmd", 1, 256, 0, False),
+    (2, "generic_smem", 1, 256, 0, False),
+    (4, "spmd", 1, 256, 0, False),
+    (4, "generic_shfl", 2, 256, 0, False),
+    (4, "generic_smem", 1, 256, 0, False),
+    (8, "spmd", 1, 256, 0, False),
+    (8, "generic_smem", 1, 256, 0, False),
+    (8, "generic_shfl", 1, 256, 0, False),
+    (16, "spmd", 2, 256, 0, False),
+    (32, "spmd", 2, 256, 0, False),
+    (32, "generic_smem", 1, 256, 0, False),
+]
+
+
+def cfg_of(c):
+    S, mode, U, T, halo, hints = c
+    return dict(simdlen=S, mode=mode, outer_unroll=U, threads_per_team=T, x_halo=halo,
+                stream_hints=hints)
+
+
+def time_steps(torch, fn, flush, P, iters, events_out=None):
+    """Per-step CUDA-event times (ms) on the current stream, L2 flushed between steps."""
+    ts = []
+    for _ in range(iters):
+        P.l2_flush(flush)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        fn()
+        e1.record()
+        ts.append((e0, e1))
+    torch.cuda.synchronize()
+    return [a.elapsed_time(b) for a, b in ts]
+
+
+def run_gpu(args, rank, world, local_rank):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_icpp_wrightdtcc23_b200 as P
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    spec = SPEC
+    if world > 1:
+        gspec = R.SpmvSpec(f"{spec.name}x{world}", spec.seed, spec.nrows * world, spec.ncols * world,
+                           spec.nnz_min, spec.nnz_max, spec.structure, spec.band_w, spec.far_den)
+        chunk, rb, nloc = P.shard_rows(gspec.nrows, world, rank)
+    else:
+        gspec, rb, nloc = spec, 0, spec.nrows
+    rp, col, val = R.spmv_matrix(gspec, row_begin=rb, nrows=nloc)
+    nnz = int(val.size)
+    pin = lambda a: torch.from_numpy(a).pin_memory()
+    h_rp, h_col, h_val = pin(rp), pin(col), pin(val)
+    d_rp, d_col, d_val = (h_rp.to(dev), h_col.to(dev), h_val.to(dev))
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)   # 4x the 126 MB L2
+    peak, peak_src = peaks()
+
+    if world == 1:
+        x = R.spmv_x(spec)
+        h_x = pin(x)
+        d_x = h_x.to(dev)
+        d_y = torch.empty(spec.nrows, dtype=torch.float64, device=dev)
+        B = alg_bytes(spec.nrows, spec.ncols, nnz)
+
+        # untimed autotune over the candidate (simdlen, mode, variant) set
+        sweep = []
+        for c in CANDIDATES:
+            cfg = cfg_of(c)
+            fn = lambda cfg=cfg: P.spmv_csr_f64(d_rp, d_col, d_val, d_x, d_y, **cfg)
+            try:
+                fn()
+            except P.NestError as e:
+                print(f"skip {c}: {e}", file=sys.stderr)
+                continue
+            ts = time_steps(torch, fn, flush, P, 5)
+            sweep.append((statistics.median(ts), c))
+        sweep.sort(key=lambda t: t[0])
+        best = sweep[0][1]
+        s1 = min((t for t in sweep if t[1][0] == 1), key=lambda t: t[0])
+        cfg = cfg_of(best)
+        step = lambda: P.spmv_csr_f64(d_rp, d_col, d_val, d_x, d_y, **cfg)
+
+        for _ in range(args.warmup):
+            step()
+        torch.cuda.synchronize()
+        # timed region: K steps, L2 flushed between steps (flush outside the events)
+        with ClockSampler(local_rank) as clk:
+            torch.cuda.synchronize()
+            ts = time_steps(torch, step, flush, P, args.steps)
+            torch.cuda.synchronize()
+        ms = sum(ts) / len(ts)
+        value = B / (ms / 1e3) / 1e9
+        # simd-folded two-level mapping (simdlen = 1), same protocol
+        s1_cfg = cfg_of(s1[1])
+        ts1 = time_steps(torch, lambda: P.spmv_csr_f64(d_rp, d_col, d_val, d_x, d_y, **s1_cfg), flush, P,
+                         max(3, args.steps // 2))
+        ms1 = sum(ts1) / len(ts1)
+
+        # e2e through the C ABI with HOST buffers: H2D of A and x, the SpMV, D2H of y
+        h_y = torch.empty(spec.nrows, dtype=torch.float64).pin_memory()
+        ws = torch.empty(P.hostio_workspace_bytes(spec.nrows, spec.ncols, nnz), dtype=torch.uint8, device=dev)
+        e2e_step = lambda: P.spmv_csr_f64_hostio(h_rp, h_col, h_val, h_x, h_y, ws, **cfg)
+        e2e_step()
+        torch.cuda.synchronize()
+        n_e2e = max(3, min(args.steps, 10))
+        te = []
+        for _ in range(n_e2e):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            e2e_step()
+            e1.record()
+            e1.synchronize()
+            te.append(e0.elapsed_time(e1))
+        ms_e2e = sum(te) / len(te)
+        h2d = (spec.nrows + 1) * 8 + nnz * 12 + spec.ncols * 8
+        d2h = spec.nrows * 8
+
+        kernel_name = (f"spmv_xwin_kernel<{best[0]},...>" if best[4] else
+                       f"nest_kernel<S={best[0]},{best[1]},SUM,U={best[2]},SpmvBody<{int(best[5])}>>")
+        traffic = None
+        try:
+            with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
+                traffic = json.load(f).get(json.dumps(list(best)))
+        except Exception:
+            pass
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": 1, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": f"{spec.name}: CSR SpMV fp64 {spec.nrows}x{spec.ncols}, nnz/row "
+                                   f"U{{{spec.nnz_min}..{spec.nnz_max}}} banded+far (W={spec.band_w}, far "
+                                   f"1/{spec.far_den}), seed {spec.seed} (BASELINE.json configs[1])",
+                       "nnz": nnz, "alg_bytes": B, "simdlen": best[0], "mode": best[1],
+                       "outer_unroll": best[2], "threads_per_team": best[3], "x_halo": best[4],
+                       "stream_hints": best[5], "l2": "flushed (512 MiB write) between timed steps",
+                       "parallelism": "1 GPU"},
+            "speedup_vs_simdlen1": ms1 / ms,
+            "simdlen1": {"ms_per_step": ms1, "GBs": B / (ms1 / 1e3) / 1e9, "config": cfg_of(s1[1])},
+            "sweep_ms": {json.dumps(list(c)): round(t, 4) for t, c in sweep},
+            "roofline": {"bound": "hbm", "achieved": value, "peak": peak, "unit": "GB/s",
+                         "frac": value / peak, "traffic": traffic, "peak_source": peak_src,
+                         "kernel": kernel_name, "frac_of_8TBs_spec": value / 8000.0},
+            "e2e": {"value": B / (ms_e2e / 1e3) / 1e9, "unit": UNIT, "h2d_bytes_per_step": h2d,
+                    "d2h_bytes_per_step": d2h, "ms_per_step": ms_e2e},
+            "gpu_launches": 2 * args.steps,
+            "gpu_launches_detail": "per step: 1 SpMV kernel + 1 l2_flush kernel (flush outside the step events)",
+            "clocks": clk.summary(),
+        }
+        if not args.no_cpu_baseline:
+            line["cpu_baseline"] = cpu_baseline(spec)
+        print(json.dumps(line), flush=True)
+        return
+
+    # ---- N > 1: row-partitioned SpMV, NCCL all-gather of x inside each step
+    comm = P.Comm()
+    xchunk = -(-gspec.ncols // world)
+    xb = min(rank * xchunk, gspec.ncols)
+    xl = R.spmv_x(gspec, begin=xb, n=min(xchunk, gspec.ncols - xb))
+    d_xl = torch.zeros(xchunk, dtype=torch.float64, device=dev)
+    d_xl[:xl.size] = torch.from_numpy(xl).to(dev)
+    d_xf = torch.empty(xchunk * world, dtype=torch.float64, device=dev)
+    d_y = torch.empty(nloc, dtype=torch.float64, device=dev)
+    cfg = dict(simdlen=4, mode="spmd", outer_unroll=1)
+    step = lambda: comm.spmv_csr_f64(gspec.nrows, gspec.ncols, d_rp, d_col, d_val, d_xl, d_xf, d_y, **cfg)
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    dist.barrier()
+    with ClockSampler(local_rank) as clk:
+        torch.cuda.synchronize()
+        ts = time_steps(torch, step, flush, P, args.steps)
+        torch.cuda.synchronize()
+    dist.barrier()
+    ms_local = sum(ts) / len(ts)
+    t = torch.tensor([ms_local], dtype=torch.float64, device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms = float(t.item())
+    nnz_t = torch.tensor([nnz], dtype=torch.int64, device=dev)
+    dist.all_reduce(nnz_t)
+    B = alg_bytes(gspec.nrows, gspec.ncols, int(nnz_t.item()))
+    if rank == 0:
+        line = {"metric": METRIC, "value": B / (ms / 1e3) / 1e9, "unit": UNIT, "n_gpus": world,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+                "config": {"workload": f"row-partitioned CSR SpMV fp64, {spec.nrows} rows per rank "
+                                       f"(global {gspec.nrows}), nnz/row U{{{spec.nnz_min}..{spec.nnz_max}}}, "
+                                       "NCCL all-gather of x each step", "parallelism": f"rows/{world}",
+                           "l2": "flushed between timed steps", **cfg},
+                "gpu_launches": 2 * args.steps, "clocks": clk.summary(), "e2e": None}
+        print(json.dumps(line), flush=True)
+    comm.close()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        import torch.distributed as dist
+        backend = "gloo" if args.impl == "reference" else "nccl"
+        if backend == "nccl":
+            import torch
+            torch.cuda.set_device(local_rank)
+        dist.init_process_group(backend)
+    try:
+        if args.impl == "reference":
+            run_reference(args, rank, world)
+        else:
+            run_gpu(args, rank, world, local_rank)
+    finally:
+        if world > 1:
+            import torch.distributed as dist
+            dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -24,6 +24,32 @@ def shard_rows(n: int, nranks: int, rank: int):
     return chunk, b, min(b + chunk, n) - b
 
 
+def x_chunk(ncols: int, nranks: int) -> int:
+    """x is all-gathered in equal chunks of ceil(ncols/P) doubles, so global
+    column j lands at x_full[j] (x_full holds P*xchunk doubles)."""
+    return -(-ncols // nranks)
+
+
+def local_x_range(ncols: int, nranks: int, rank: int):
+    """(begin, count) of the slice of x that rank owns; the tail rank pads."""
+    xc = x_chunk(ncols, nranks)
+    b = min(rank * xc, ncols)
+    return b, min(xc, ncols - b)
+
+
+def broadcast_unique_id(group=None) -> bytes:
+    """Rank 0 creates the 128-byte NCCL unique id inside libnest.so; the torch
+    process group (any backend) broadcasts it to every rank."""
+    import torch.distributed as dist
+    uid = (ctypes.c_uint8 * 128)()
+    if dist.get_rank(group) == 0:
+        check(N.nest_comm_unique_id(uid), "nest_comm_unique_id")
+    obj = [bytes(uid)]
+    src = 0 if group is None else dist.get_global_rank(group, 0)
+    dist.broadcast_object_list(obj, src=src, group=group)
+    return obj[0]
+
+
 class Comm:
     """A libnest-owned NCCL communicator over the ranks of a torch process group."""
 
@@ -32,12 +58,7 @@ class Comm:
         import torch.distributed as dist
         self.rank = dist.get_rank(group)
         self.nranks = dist.get_world_size(group)
-        uid = (ctypes.c_uint8 * 128)()
-        if self.rank == 0:
-            check(N.nest_comm_unique_id(uid), "nest_comm_unique_id")
-        obj = [bytes(uid)]
-        dist.broadcast_object_list(obj, src=0, group=group)
-        uid = (ctypes.c_uint8 * 128).from_buffer_copy(obj[0])
+        uid = (ctypes.c_uint8 * 128).from_buffer_copy(broadcast_unique_id(group))
         self._h = ctypes.c_void_p()
         check(N.nest_comm_init(uid, self.nranks, self.rank, ctypes.byref(self._h)), "nest_comm_init")
         self._torch = torch
@@ -59,7 +80,7 @@ class Comm:
         torch = self._torch
         nrows_local = rowptr.numel() - 1
         nnz = val.numel()
-        xchunk = -(-ncols_global // self.nranks)
+        xchunk = x_chunk(ncols_global, self.nranks)
         if y_local is None:
             y_local = torch.empty(nrows_local, dtype=torch.float64, device=val.device)
         d = make_desc(**cfg)
