@@ -84,7 +84,14 @@ enum {
     NEST_F_PERSISTENT_GRID = 1u << 0,
     /* stream the CSR arrays with L2 evict-first / L1 no-allocate hints and
      * keep x cached (SpMV only; results unchanged). */
-    NEST_F_STREAM_HINTS = 1u << 1
+    NEST_F_STREAM_HINTS = 1u << 1,
+    /* SpMV only: warp-specialised pipeline.  Warp 0 of each team stages the
+     * team's row chunks (rowptr, colind, val and, with x_halo > 0, the x
+     * window) into shared memory with bulk asynchronous copies (TMA engine) and
+     * mbarriers; warps 1.. run the loop nest out of shared memory.  Needs
+     * threads_per_team >= 64 and 16-byte aligned colind, val and x.  Results
+     * are identical to the unstaged path. */
+    NEST_F_STAGED = 1u << 2
 };
 
 /* The nest descriptor: team, thread and simd extents, mode and reduction.

@@ -157,7 +157,9 @@ int oracle_simd_owner(int64_t trip, int32_t S, int32_t *owner) {
  * power of two dividing the warp (groups equal-size, never spanning a warp:
  * PAPER.md:484-491, 511-513, 689-691) and T is whole warps in [32,1024].
  * groups/team G = T/S; the sharing space (default 2048 B)
- * is divided evenly among the groups: slot = sharing/G;
+ * is divided evenly among the groups: slot = sharing/G
+ * rounded down to the 8-byte alignment of the payload entries (the paper's
+ * entries are pointers; R8);
  * a payload larger than its slot falls back to global memory
  * (PAPER.md:680-684).  out = {G, slot_bytes, uses_global_fallback}. */
 int oracle_plan_geometry(int32_t T, int32_t S, int32_t sharing_bytes, int32_t payload_bytes,
@@ -167,7 +169,7 @@ int oracle_plan_geometry(int32_t T, int32_t S, int32_t sharing_bytes, int32_t pa
     if (!s_ok || T < 32 || T > 1024 || T % 32 || sharing_bytes < 0 || payload_bytes < 0) return 1;
     int32_t G = T / S;
     out[0] = G;
-    out[1] = sharing_bytes / G;
+    out[1] = (sharing_bytes / G) / 8 * 8;   /* each slot holds 8-byte aligned payloads (R8) */
     out[2] = payload_bytes > out[1];
     return 0;
 }

@@ -3,6 +3,7 @@
 #include <cuda_runtime.h>
 
 #include <climits>
+#include <cstdint>
 #include <cstdarg>
 #include <cstdio>
 #include <mutex>
@@ -70,14 +71,14 @@ static nest_status validate_desc(const nest_desc* d, int32_t* T, int32_t* sharin
     *U = d->outer_unroll ? d->outer_unroll : 1;
     if (*U != 1 && *U != 2 && *U != 4)
         return fail(NEST_ERR_INVALID_ARG, "outer_unroll %d: need 1, 2 or 4", d->outer_unroll);
-    if (d->flags & ~(uint32_t)(NEST_F_PERSISTENT_GRID | NEST_F_STREAM_HINTS))
+    if (d->flags & ~(uint32_t)(NEST_F_PERSISTENT_GRID | NEST_F_STREAM_HINTS | NEST_F_STAGED))
         return fail(NEST_ERR_INVALID_ARG, "unknown flags 0x%x", d->flags);
     if (d->reserved[0] || d->reserved[1])
         return fail(NEST_ERR_INVALID_ARG, "reserved fields must be 0");
     return NEST_OK;
 }
 
-static nest_status resident_blocks(int32_t T, int32_t smem, int64_t* out) {
+nest_status resident_blocks(int32_t T, int32_t smem, int64_t* out) {
     int sms = 0;
     nest_status s = sm_count(&sms);
     if (s != NEST_OK) return s;
@@ -97,6 +98,10 @@ static nest_status plan_core(const nest_desc* d, int64_t outer, int32_t K, int32
     if (d->x_halo < 0) return fail(NEST_ERR_INVALID_ARG, "x_halo %d < 0", d->x_halo);
     if (d->x_halo > 0 && !spmv_window)
         return fail(NEST_ERR_INVALID_ARG, "x_halo applies to the CSR SpMV only");
+    if ((d->flags & NEST_F_STAGED) && !spmv_window)
+        return fail(NEST_ERR_INVALID_ARG, "NEST_F_STAGED applies to the CSR SpMV only");
+    if ((d->flags & NEST_F_STAGED) && T < 64)
+        return fail(NEST_ERR_INVALID_ARG, "NEST_F_STAGED needs threads_per_team >= 64 (producer + consumer warps)");
     if (K <= 0) K = 1;
     const int32_t S = d->simdlen;
     const bool smem_mode = d->mode == NEST_MODE_GENERIC_SMEM && S > 1;
@@ -106,7 +111,7 @@ static nest_status plan_core(const nest_desc* d, int64_t outer, int32_t K, int32
     q.mode = S == 1 ? NEST_MODE_SPMD : d->mode;
     q.reduce = d->reduce;
     q.groups = T / S;
-    q.slot_bytes = sharing / q.groups;                  // split evenly
+    q.slot_bytes = (sharing / q.groups) & ~7;           // split evenly, 8-B aligned (R8)
     q.payload_bytes = payload;
     q.fallback = smem_mode && payload > q.slot_bytes;
     q.unroll = U;
@@ -117,7 +122,10 @@ static nest_status plan_core(const nest_desc* d, int64_t outer, int32_t K, int32
     const int64_t per_group = (U + K - 1) / K;
     const int64_t denom = (int64_t)q.groups * per_group;
     int64_t needed = (outer + denom - 1) / denom;
-    if (d->x_halo > 0) {
+    if (d->flags & NEST_F_STAGED) {
+        q.x_halo = d->x_halo;   // stage sizes and grid: plan_spmv_staged (needs nnz)
+        q.grid = d->num_teams;
+    } else if (d->x_halo > 0) {
         // x window (spmv_xwin.cuh): ring of 2^k >= 2R + 2H doubles, R = G*U rows per chunk,
         // plus a double-buffered rowptr stage; always a persistent block schedule.
         const int64_t R = (int64_t)q.groups * U;
@@ -284,8 +292,15 @@ NEST_API nest_status nest_spmv_csr_f64(const nest_desc* desc, int64_t nrows, int
     if (nrows == 0) return NEST_OK;
     if (!rowptr || !y) return fail(NEST_ERR_INVALID_ARG, "rowptr/y is NULL");
     if (nnz > 0 && (!colind || !val || !x)) return fail(NEST_ERR_INVALID_ARG, "colind/val/x is NULL");
+    const bool staged = (p.flags & NEST_F_STAGED) != 0;
+    if (staged && (s = plan_spmv_staged(&p, nrows, nnz, desc->sharing_bytes ? desc->sharing_bytes : kDefaultSharing)) != NEST_OK)
+        return s;
+    if (staged && ((reinterpret_cast<uintptr_t>(colind) | reinterpret_cast<uintptr_t>(val) |
+                    reinterpret_cast<uintptr_t>(x)) & 15))
+        return fail(NEST_ERR_UNSUPPORTED, "NEST_F_STAGED needs 16-byte aligned colind, val and x");
     unsigned char* fb = nullptr;
     if ((s = prepare_fallback(p, &fb)) != NEST_OK) return s;
+    if (staged) return launch_spmv_staged(p, nrows, ncols, nnz, rowptr, colind, val, x, y, fb, as_stream(stream));
     if (p.x_halo > 0) return launch_spmv_xwin(p, nrows, ncols, rowptr, colind, val, x, y, fb, as_stream(stream));
     return launch_spmv(p, (p.flags & NEST_F_STREAM_HINTS) != 0, nrows, rowptr, colind, val, x, y, fb,
                        as_stream(stream));
@@ -324,6 +339,9 @@ NEST_API nest_status nest_spmv_csr_f64_hostio(const nest_desc* desc, int64_t nro
     double* d_x = reinterpret_cast<double*>(w);
     w += align256((size_t)ncols * 8);
     double* d_y = reinterpret_cast<double*>(w);
+    const bool staged = (p.flags & NEST_F_STAGED) != 0;
+    if (staged && (s = plan_spmv_staged(&p, nrows, nnz, desc->sharing_bytes ? desc->sharing_bytes : kDefaultSharing)) != NEST_OK)
+        return s;
     unsigned char* fb = nullptr;
     if ((s = prepare_fallback(p, &fb)) != NEST_OK) return s;
     cudaStream_t st = as_stream(stream);
@@ -333,7 +351,8 @@ NEST_API nest_status nest_spmv_csr_f64_hostio(const nest_desc* desc, int64_t nro
         (nnz && (e = cudaMemcpyAsync(d_val, h_val, (size_t)nnz * 8, cudaMemcpyHostToDevice, st))) ||
         (ncols && (e = cudaMemcpyAsync(d_x, h_x, (size_t)ncols * 8, cudaMemcpyHostToDevice, st))))
         return cuda_fail(e, "host->device copy");
-    s = p.x_halo > 0 ? launch_spmv_xwin(p, nrows, ncols, d_rowptr, d_col, d_val, d_x, d_y, fb, st)
+    s = staged ? launch_spmv_staged(p, nrows, ncols, nnz, d_rowptr, d_col, d_val, d_x, d_y, fb, st)
+        : p.x_halo > 0 ? launch_spmv_xwin(p, nrows, ncols, d_rowptr, d_col, d_val, d_x, d_y, fb, st)
                      : launch_spmv(p, (p.flags & NEST_F_STREAM_HINTS) != 0, nrows, d_rowptr, d_col, d_val,
                                    d_x, d_y, fb, st);
     if (s != NEST_OK) return s;

@@ -29,6 +29,10 @@ struct Plan {
     int64_t outer = 0;
     int32_t x_halo = 0;    // SpMV x window half-width (0 = none)
     int32_t xw_log2 = 0;   // ring of 2^xw_log2 doubles
+    // NEST_F_STAGED pipeline (spmv_staged.cuh)
+    int32_t xw = 0;        // x ring capacity in doubles (even; 0 = no window)
+    int32_t nb = 0;        // stage capacity in nonzeros
+    int32_t ns = 0;        // stages in flight
 };
 
 // Record a thread-local error message and return `s`.
@@ -62,6 +66,12 @@ nest_status launch_spmv(const Plan& p, bool hints, int64_t nrows, const int64_t*
 nest_status launch_spmv_xwin(const Plan& p, int64_t nrows, int64_t ncols, const int64_t* rowptr,
                              const int32_t* col, const double* val, const double* x, double* y,
                              unsigned char* fb, cudaStream_t st);
+// NEST_F_STAGED: finish the plan from the matrix shape (stage sizes, grid) and launch.
+nest_status plan_spmv_staged(Plan* p, int64_t nrows, int64_t nnz, int32_t sharing_bytes);
+nest_status launch_spmv_staged(const Plan& p, int64_t nrows, int64_t ncols, int64_t nnz,
+                               const int64_t* rowptr, const int32_t* col, const double* val,
+                               const double* x, double* y, unsigned char* fb, cudaStream_t st);
+nest_status resident_blocks(int32_t T, int32_t smem, int64_t* out);
 nest_status launch_batched(const Plan& p, int64_t batch, int32_t m, int32_t n, const float* A,
                            const float* x, float* y, unsigned char* fb, cudaStream_t st);
 nest_status launch_stencil(const Plan& p, int64_t nouter, int32_t L, const double* in,

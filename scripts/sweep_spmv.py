@@ -25,6 +25,7 @@ def main():
     ap.add_argument("--hints", default="0,1")
     ap.add_argument("--threads", default="256")
     ap.add_argument("--halos", default="0")
+    ap.add_argument("--staged", default="0")
     ap.add_argument("--out", default=None)
     a = ap.parse_args()
     spec = getattr(R, a.spec)
@@ -44,9 +45,10 @@ def main():
                 if S == 1 and mode != "spmd":
                     continue
                 for U in map(int, a.unrolls.split(",")):
-                    for h, xh in [(h, xh) for h in map(int, a.hints.split(",")) for xh in map(int, a.halos.split(","))]:
+                    for h, xh, sg in [(h, xh, sg) for h in map(int, a.hints.split(",")) for xh in map(int, a.halos.split(","))
+                                      for sg in map(int, a.staged.split(","))]:
                         cfg = dict(simdlen=S, mode=mode, outer_unroll=U, stream_hints=bool(h), threads_per_team=T,
-                                   x_halo=xh)
+                                   x_halo=xh, staged=bool(sg))
                         try:
                             P.spmv_csr_f64(*t, y, **cfg)
                         except P.NestError as e:
@@ -64,7 +66,7 @@ def main():
                             e1.synchronize()
                             ts.append(e0.elapsed_time(e1))
                         ms = float(np.median(ts))
-                        r = dict(T=T, S=S, mode=mode, U=U, hints=h, halo=xh, ms=ms, min_ms=min(ts), GBs=B / ms / 1e6)
+                        r = dict(T=T, S=S, mode=mode, U=U, hints=h, halo=xh, staged=sg, ms=ms, min_ms=min(ts), GBs=B / ms / 1e6)
                         res.append(r)
                         print(json.dumps(r), flush=True)
     best = min(res, key=lambda r: r["ms"])

@@ -341,3 +341,65 @@ def test_spmv_xwin_too_big_is_unsupported(P, cfg1):
         P.spmv_csr_f64(dev(rp), dev(col), dev(val), dev(x), simdlen=1, threads_per_team=1024,
                        outer_unroll=4, x_halo=20000)
     assert e.value.status == 2
+
+
+# ------------------------------------------------------------------ a8 SpMV, staged pipeline
+@pytest.mark.parametrize("S", SIMDLENS)
+@pytest.mark.parametrize("mode", MODES)
+def test_spmv_staged(P, banded, S, mode):
+    for values in ("int", "real"):
+        rp, col, val, x, yref, aref = banded[values]
+        t = [dev(rp), dev(col), dev(val), dev(x)]
+        for halo, U, T, teams in ((0, 1, 256, 0), (700, 1, 1024, 0), (64, 2, 512, 0), (4096, 4, 128, 0),
+                                  (1, 2, 64, 0), (700, 1, 256, 3), (300, 4, 1024, 1)):
+            if (T - 32) // S == 0:
+                continue
+            y = host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, outer_unroll=U, threads_per_team=T,
+                                    x_halo=halo, num_teams=teams, staged=True))
+            if values == "int":
+                assert np.array_equal(bits(y), bits(yref)), (halo, U, T, teams)
+            else:
+                assert_close(y, yref, aref, 1e-12)
+
+
+def test_spmv_staged_long_rows_and_odd_sizes(P):
+    # rows longer than any stage (global path), odd nnz / ncols (unaligned tails)
+    for lens, ncols in (([0, 3, 40000, 7, 1, 0, 25000, 5] * 3 + [1], 60001),
+                        ([1] * 999 + [2], 1001), ([0] * 50, 7)):
+        rp, col, val, x = _rows_matrix(lens, ncols, 11)
+        yref, _ = oracle.spmv_csr_f64(rp, col, val, x)
+        t = [dev(rp), dev(col), dev(val), dev(x)]
+        for S in (1, 4, 32):
+            for mode in MODES:
+                for halo in (0, 3, 1000):
+                    y = host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, x_halo=halo, staged=True,
+                                            threads_per_team=256))
+                    assert np.array_equal(bits(y), bits(yref)), (lens[:3], S, mode, halo)
+
+
+def test_spmv_staged_cfg2_full_size_sampled(P):
+    spec = R.CFG2
+    rp, col, val = R.spmv_matrix(spec)
+    x = R.spmv_x(spec)
+    t = [dev(rp), dev(col), dev(val), dev(x)]
+    rng = np.random.default_rng(8)
+    starts = np.concatenate([[0, spec.nrows - 64], rng.integers(0, spec.nrows - 64, 20)])
+    ref = {int(s): oracle.spmv_csr_f64(*R.spmv_matrix(spec, row_begin=int(s), nrows=64), x) for s in starts}
+    for S, mode, U, T, halo in ((8, "spmd", 2, 1024, 4096), (4, "generic_smem", 2, 512, 4096),
+                                (16, "generic_shfl", 1, 1024, 4096), (1, "spmd", 1, 256, 4096),
+                                (8, "spmd", 1, 1024, 0)):
+        y = host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, outer_unroll=U, threads_per_team=T,
+                                x_halo=halo, staged=True))
+        for s, (yr, ar) in ref.items():
+            assert_close(y[s:s + 64], yr, ar, 1e-12)
+
+
+def test_spmv_staged_alignment_and_small_team(P, cfg1):
+    rp, col, val, x, _, _ = cfg1["int"]
+    dcol = torch.from_numpy(np.concatenate([[0], col]).astype(np.int32)).cuda()[1:]
+    with pytest.raises(P.NestError) as e:
+        P.spmv_csr_f64(dev(rp), dcol, dev(val), dev(x), staged=True)
+    assert e.value.status == 2
+    with pytest.raises(P.NestError) as e:
+        P.spmv_csr_f64(dev(rp), dev(col), dev(val), dev(x), staged=True, threads_per_team=32)
+    assert e.value.status == 1

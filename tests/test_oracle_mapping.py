@@ -107,3 +107,13 @@ def test_shard_partition_covers(n, P):
         assert b == seen or cnt == 0
         seen += cnt
     assert seen == n
+
+
+def test_sharing_slots_are_8_byte_aligned_even_split():
+    # DESIGN.md R8: sharing/G rounded down to the 8-byte payload alignment
+    assert oracle.plan_geometry(256, 8, 1000, 24) == (32, 24, 0)      # 1000/32 = 31.25 -> 24
+    assert oracle.plan_geometry(1024, 2, 2048, 24) == (512, 0, 1)     # 4 B -> 0: fallback
+    for T in (64, 256, 1024):
+        for S in (2, 4, 8, 16, 32):
+            G, slot, _ = oracle.plan_geometry(T, S, 2048, 0)
+            assert slot % 8 == 0 and G * slot <= 2048 and G * (slot + 8) > 2048 - 8 * G
