@@ -154,28 +154,33 @@ def run_reference(args, rank, world):
 
 
 # ---------------------------------------------------------------- GPU arm
+# (simdlen, mode, outer_unroll, threads_per_team, x_halo, flags) -- flags: "b" blocked
+# team schedule, "s" staged pipeline, "h" streaming cache hints
 CANDIDATES = [
-    # (simdlen, mode, outer_unroll, threads, x_halo, stream_hints)
-    (1, "spmd", 1, 256, 0, False),
-    (1, "spmd", 2, 256, 0, False),
-    (2, "spmd", 1, 256, 0, False),
-    (2, "generic_smem", 1, 256, 0, False),
-    (4, "spmd", 1, 256, 0, False),
-    (4, "generic_shfl", 2, 256, 0, False),
-    (4, "generic_smem", 1, 256, 0, False),
-    (8, "spmd", 1, 256, 0, False),
-    (8, "generic_smem", 1, 256, 0, False),
-    (8, "generic_shfl", 1, 256, 0, False),
-    (16, "spmd", 2, 256, 0, False),
-    (32, "spmd", 2, 256, 0, False),
-    (32, "generic_smem", 1, 256, 0, False),
+    (1, "spmd", 1, 256, 0, ""),
+    (1, "spmd", 1, 1024, 0, "b"),
+    (2, "spmd", 1, 1024, 0, "b"),
+    (2, "generic_smem", 1, 1024, 0, "b"),
+    (2, "generic_shfl", 1, 1024, 0, "b"),
+    (4, "spmd", 1, 1024, 0, "b"),
+    (4, "generic_smem", 1, 1024, 0, "b"),
+    (4, "generic_shfl", 1, 1024, 0, "b"),
+    (8, "spmd", 1, 1024, 0, "b"),
+    (8, "generic_smem", 1, 1024, 0, "b"),
+    (16, "spmd", 1, 1024, 0, "b"),
+    (32, "spmd", 1, 1024, 0, "b"),
+    (2, "spmd", 1, 256, 0, ""),
+    (4, "spmd", 1, 256, 0, ""),
+    (8, "spmd", 1, 256, 0, ""),
+    (4, "spmd", 1, 512, 4096, "s"),
+    (2, "spmd", 1, 1024, 4096, "s"),
 ]
 
 
 def cfg_of(c):
-    S, mode, U, T, halo, hints = c
+    S, mode, U, T, halo, fl = c
     return dict(simdlen=S, mode=mode, outer_unroll=U, threads_per_team=T, x_halo=halo,
-                stream_hints=hints)
+                stream_hints="h" in fl, staged="s" in fl, blocked="b" in fl)
 
 
 def time_steps(torch, fn, flush, P, iters, events_out=None):
@@ -236,7 +241,7 @@ def run_gpu(args, rank, world, local_rank):
             sweep.append((statistics.median(ts), c))
         sweep.sort(key=lambda t: t[0])
         best = sweep[0][1]
-        s1 = min((t for t in sweep if t[1][0] == 1), key=lambda t: t[0])
+        s1 = min((t for t in sweep if t[1][0] == 1), key=lambda t: t[0])   # best 2-level (simdlen 1)
         cfg = cfg_of(best)
         step = lambda: P.spmv_csr_f64(d_rp, d_col, d_val, d_x, d_y, **cfg)
 
@@ -275,8 +280,8 @@ def run_gpu(args, rank, world, local_rank):
         h2d = (spec.nrows + 1) * 8 + nnz * 12 + spec.ncols * 8
         d2h = spec.nrows * 8
 
-        kernel_name = (f"spmv_xwin_kernel<{best[0]},...>" if best[4] else
-                       f"nest_kernel<S={best[0]},{best[1]},SUM,U={best[2]},SpmvBody<{int(best[5])}>>")
+        kernel_name = (f"spmv_staged_kernel<S={best[0]},{best[1]},SUM,U={best[2]}>" if "s" in best[5] else
+                       f"nest_kernel<S={best[0]},{best[1]},SUM,U={best[2]},SpmvBody<{int('h' in best[5])}>>")
         traffic = None
         try:
             with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
@@ -292,7 +297,9 @@ def run_gpu(args, rank, world, local_rank):
                                    f"1/{spec.far_den}), seed {spec.seed} (BASELINE.json configs[1])",
                        "nnz": nnz, "alg_bytes": B, "simdlen": best[0], "mode": best[1],
                        "outer_unroll": best[2], "threads_per_team": best[3], "x_halo": best[4],
-                       "stream_hints": best[5], "l2": "flushed (512 MiB write) between timed steps",
+                       "variant": {"": "cyclic teams", "b": "blocked teams", "s": "staged pipeline",
+                                   "h": "stream hints"}.get(best[5], best[5]),
+                       "l2": "flushed (512 MiB write) between timed steps",
                        "parallelism": "1 GPU"},
             "speedup_vs_simdlen1": ms1 / ms,
             "simdlen1": {"ms_per_step": ms1, "GBs": B / (ms1 / 1e3) / 1e9, "config": cfg_of(s1[1])},

@@ -88,10 +88,17 @@ enum {
     /* SpMV only: warp-specialised pipeline.  Warp 0 of each team stages the
      * team's row chunks (rowptr, colind, val and, with x_halo > 0, the x
      * window) into shared memory with bulk asynchronous copies (TMA engine) and
-     * mbarriers; warps 1.. run the loop nest out of shared memory.  Needs
-     * threads_per_team >= 64 and 16-byte aligned colind, val and x.  Results
-     * are identical to the unstaged path. */
-    NEST_F_STAGED = 1u << 2
+     * mbarriers; warps 1-2 gather x for the staged nonzeros (window hits from
+     * shared memory, the rest with asynchronous copies); warps 3.. run the loop
+     * nest out of shared memory.  Needs threads_per_team >= 128 and 16-byte
+     * aligned colind, val and x.  Results are identical to the unstaged path. */
+    NEST_F_STAGED = 1u << 2,
+    /* "teams distribute" with a static block schedule: team b owns the
+     * contiguous outer range [b*C, (b+1)*C) and its SIMD groups take it
+     * cyclically, so the rows in flight on an SM are neighbours (x stays in
+     * L1/L2 for banded matrices).  Implies a persistent grid.  Results are
+     * identical (the schedule never changes a row's arithmetic). */
+    NEST_F_BLOCKED = 1u << 3
 };
 
 /* The nest descriptor: team, thread and simd extents, mode and reduction.

@@ -25,6 +25,7 @@ NEST_REDUCE_SUM, NEST_REDUCE_MAX, NEST_REDUCE_MIN = 0, 1, 2
 NEST_F_PERSISTENT_GRID = 1 << 0
 NEST_F_STREAM_HINTS = 1 << 1
 NEST_F_STAGED = 1 << 2
+NEST_F_BLOCKED = 1 << 3
 
 
 class nest_desc(ctypes.Structure):

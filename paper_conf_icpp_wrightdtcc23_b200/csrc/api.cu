@@ -71,7 +71,7 @@ static nest_status validate_desc(const nest_desc* d, int32_t* T, int32_t* sharin
     *U = d->outer_unroll ? d->outer_unroll : 1;
     if (*U != 1 && *U != 2 && *U != 4)
         return fail(NEST_ERR_INVALID_ARG, "outer_unroll %d: need 1, 2 or 4", d->outer_unroll);
-    if (d->flags & ~(uint32_t)(NEST_F_PERSISTENT_GRID | NEST_F_STREAM_HINTS | NEST_F_STAGED))
+    if (d->flags & ~(uint32_t)(NEST_F_PERSISTENT_GRID | NEST_F_STREAM_HINTS | NEST_F_STAGED | NEST_F_BLOCKED))
         return fail(NEST_ERR_INVALID_ARG, "unknown flags 0x%x", d->flags);
     if (d->reserved[0] || d->reserved[1])
         return fail(NEST_ERR_INVALID_ARG, "reserved fields must be 0");
@@ -100,8 +100,9 @@ static nest_status plan_core(const nest_desc* d, int64_t outer, int32_t K, int32
         return fail(NEST_ERR_INVALID_ARG, "x_halo applies to the CSR SpMV only");
     if ((d->flags & NEST_F_STAGED) && !spmv_window)
         return fail(NEST_ERR_INVALID_ARG, "NEST_F_STAGED applies to the CSR SpMV only");
-    if ((d->flags & NEST_F_STAGED) && T < 64)
-        return fail(NEST_ERR_INVALID_ARG, "NEST_F_STAGED needs threads_per_team >= 64 (producer + consumer warps)");
+    if ((d->flags & NEST_F_STAGED) && T < 128)
+        return fail(NEST_ERR_INVALID_ARG,
+                    "NEST_F_STAGED needs threads_per_team >= 128 (producer, 2 gather and >= 1 consumer warps)");
     if (K <= 0) K = 1;
     const int32_t S = d->simdlen;
     const bool smem_mode = d->mode == NEST_MODE_GENERIC_SMEM && S > 1;
@@ -150,7 +151,7 @@ static nest_status plan_core(const nest_desc* d, int64_t outer, int32_t K, int32
         }
     } else if (d->num_teams > 0) {
         q.grid = d->num_teams;
-    } else if ((d->flags & NEST_F_PERSISTENT_GRID) || q.fallback) {
+    } else if ((d->flags & (NEST_F_PERSISTENT_GRID | NEST_F_BLOCKED)) || q.fallback) {
         int64_t resident = 0;
         nest_status s = resident_blocks(T, q.smem_bytes, &resident);
         if (s != NEST_OK) return s;

@@ -40,6 +40,7 @@ struct SpmvBody {
     struct Step {
         int64_t i;
     };
+    static constexpr bool kPrefetch = false;  // software-pipelined prologue (costs registers: occupancy)
     static constexpr bool kTeamState = false;
     struct TeamShared {
         int unused;
@@ -84,6 +85,7 @@ struct BatchedBody {
     struct Step {
         int64_t out;     // b*m + r
     };
+    static constexpr bool kPrefetch = false;  // software-pipelined prologue (costs registers: occupancy)
     static constexpr bool kTeamState = false;
     struct TeamShared {
         int unused;
@@ -125,6 +127,7 @@ struct StencilBody {
         double scale;
         int64_t skip;
     };
+    static constexpr bool kPrefetch = false;  // the prologue has a side effect (visits)
     static constexpr bool kTeamState = true;
     struct TeamShared {
         unsigned long long visits;
@@ -177,6 +180,7 @@ struct ProbeBody {
     struct Step {
         int64_t i;
     };
+    static constexpr bool kPrefetch = false;  // software-pipelined prologue (costs registers: occupancy)
     static constexpr bool kTeamState = false;
     struct TeamShared {
         int unused;

@@ -21,7 +21,13 @@
 namespace nest {
 namespace cg = cooperative_groups;
 
-template <int S>
+// WU ("warp-uniform"): the caller guarantees that every lane of the warp
+// reaches each collective of the group together (all groups of the warp run
+// the same number of batches), so the data exchanges can use the full-warp
+// mask -- xor offsets < S never leave the group, results are identical --
+// and skip the sub-warp convergence checks.  Synchronisation keeps the group
+// mask (simdmask).
+template <int S, bool WU = false>
 struct SimdGroup {
     static_assert(S == 1 || S == 2 || S == 4 || S == 8 || S == 16 || S == 32,
                   "simdlen must divide the warp (PAPER.md:484-491)");
@@ -42,17 +48,33 @@ struct SimdGroup {
         }
     }
     __device__ __forceinline__ void sync() const {                                         // synchronizeWarp
-        if (S > 1) tile.sync();
+        if constexpr (S == 1) {
+            return;
+        } else if constexpr (WU) {
+            __syncwarp();   // every lane of the warp is here: the group barrier is implied
+        } else {
+            tile.sync();
+        }
     }
     template <class T>
     __device__ __forceinline__ T bcast(T v) const {                                       // lane 0 -> group
-        if (S == 1) return v;
-        return tile.shfl(v, 0);
+        if constexpr (S == 1) {
+            return v;
+        } else if constexpr (WU) {
+            return __shfl_sync(0xffffffffu, v, 0, S);
+        } else {
+            return tile.shfl(v, 0);
+        }
     }
     template <class T>
     __device__ __forceinline__ T shfl_xor(T v, unsigned m) const {
-        if (S == 1) return v;
-        return tile.shfl_xor(v, m);
+        if constexpr (S == 1) {
+            return v;
+        } else if constexpr (WU) {
+            return __shfl_xor_sync(0xffffffffu, v, m);
+        } else {
+            return tile.shfl_xor(v, m);
+        }
     }
 };
 

@@ -12,8 +12,8 @@ namespace nest {
 
 template <class Body, int U, int S, int MODE, int OP>
 nest_status launch_one(const Plan& p, const Body& body, unsigned char* fb, cudaStream_t st) {
-    nest_kernel<S, MODE, OP, U, Body><<<p.grid, p.block, p.smem_bytes, st>>>(body, p.outer,
-                                                                              p.slot_bytes, fb);
+    nest_kernel<S, MODE, OP, U, Body><<<p.grid, p.block, p.smem_bytes, st>>>(
+        body, p.outer, p.slot_bytes, fb, (p.flags & NEST_F_BLOCKED) ? 1 : 0);
     const cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e, "kernel launch");
     return NEST_OK;

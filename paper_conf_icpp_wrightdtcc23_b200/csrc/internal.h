@@ -33,6 +33,7 @@ struct Plan {
     int32_t xw = 0;        // x ring capacity in doubles (even; 0 = no window)
     int32_t nb = 0;        // stage capacity in nonzeros
     int32_t ns = 0;        // stages in flight
+    int32_t rmax = 0;      // rows per chunk at most
 };
 
 // Record a thread-local error message and return `s`.

@@ -26,6 +26,7 @@ def main():
     ap.add_argument("--threads", default="256")
     ap.add_argument("--halos", default="0")
     ap.add_argument("--staged", default="0")
+    ap.add_argument("--blocked", default="0")
     ap.add_argument("--out", default=None)
     a = ap.parse_args()
     spec = getattr(R, a.spec)
@@ -45,10 +46,11 @@ def main():
                 if S == 1 and mode != "spmd":
                     continue
                 for U in map(int, a.unrolls.split(",")):
-                    for h, xh, sg in [(h, xh, sg) for h in map(int, a.hints.split(",")) for xh in map(int, a.halos.split(","))
-                                      for sg in map(int, a.staged.split(","))]:
+                    for h, xh, sg, bl in [(h, xh, sg, bl) for h in map(int, a.hints.split(","))
+                                          for xh in map(int, a.halos.split(",")) for sg in map(int, a.staged.split(","))
+                                          for bl in map(int, a.blocked.split(","))]:
                         cfg = dict(simdlen=S, mode=mode, outer_unroll=U, stream_hints=bool(h), threads_per_team=T,
-                                   x_halo=xh, staged=bool(sg))
+                                   x_halo=xh, staged=bool(sg), blocked=bool(bl))
                         try:
                             P.spmv_csr_f64(*t, y, **cfg)
                         except P.NestError as e:
@@ -66,7 +68,7 @@ def main():
                             e1.synchronize()
                             ts.append(e0.elapsed_time(e1))
                         ms = float(np.median(ts))
-                        r = dict(T=T, S=S, mode=mode, U=U, hints=h, halo=xh, staged=sg, ms=ms, min_ms=min(ts), GBs=B / ms / 1e6)
+                        r = dict(T=T, S=S, mode=mode, U=U, hints=h, halo=xh, staged=sg, blocked=bl, ms=ms, min_ms=min(ts), GBs=B / ms / 1e6)
                         res.append(r)
                         print(json.dumps(r), flush=True)
     best = min(res, key=lambda r: r["ms"])

@@ -351,8 +351,8 @@ def test_spmv_staged(P, banded, S, mode):
         rp, col, val, x, yref, aref = banded[values]
         t = [dev(rp), dev(col), dev(val), dev(x)]
         for halo, U, T, teams in ((0, 1, 256, 0), (700, 1, 1024, 0), (64, 2, 512, 0), (4096, 4, 128, 0),
-                                  (1, 2, 64, 0), (700, 1, 256, 3), (300, 4, 1024, 1)):
-            if (T - 32) // S == 0:
+                                  (1, 2, 128, 0), (700, 1, 256, 3), (300, 4, 1024, 1)):
+            if (T - 96) // S == 0:
                 continue
             y = host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, outer_unroll=U, threads_per_team=T,
                                     x_halo=halo, num_teams=teams, staged=True))
@@ -401,5 +401,28 @@ def test_spmv_staged_alignment_and_small_team(P, cfg1):
         P.spmv_csr_f64(dev(rp), dcol, dev(val), dev(x), staged=True)
     assert e.value.status == 2
     with pytest.raises(P.NestError) as e:
-        P.spmv_csr_f64(dev(rp), dev(col), dev(val), dev(x), staged=True, threads_per_team=32)
+        P.spmv_csr_f64(dev(rp), dev(col), dev(val), dev(x), staged=True, threads_per_team=96)
     assert e.value.status == 1
+
+
+# ------------------------------------------------------------------ a8 SpMV, blocked team schedule
+@pytest.mark.parametrize("S", SIMDLENS)
+@pytest.mark.parametrize("mode", MODES)
+def test_spmv_blocked(P, banded, S, mode):
+    for values in ("int", "real"):
+        rp, col, val, x, yref, aref = banded[values]
+        t = [dev(rp), dev(col), dev(val), dev(x)]
+        for U, T, teams in ((1, 1024, 0), (2, 256, 0), (4, 512, 7), (1, 64, 1)):
+            y = host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, outer_unroll=U, threads_per_team=T,
+                                    num_teams=teams, blocked=True))
+            if values == "int":
+                assert np.array_equal(bits(y), bits(yref)), (U, T, teams)
+            else:
+                assert_close(y, yref, aref, 1e-12)
+    # stencil and batched under the blocked schedule too (the flag is generic)
+    N, L = 3001, 8
+    inp, coef, w = R.stencil_inputs(N, L, values="int")
+    yref, _, _ = oracle.nested_stencil_f64(inp, coef, w, N, L)
+    visits = torch.zeros(1, dtype=torch.int64, device="cuda")
+    y = host(P.nested_stencil_f64(dev(inp), dev(coef), dev(w), N, L, visits=visits, simdlen=S, mode=mode, blocked=True))
+    assert np.array_equal(bits(y), bits(yref)) and int(visits.item()) == N
