@@ -304,7 +304,7 @@ NEST_API nest_status nest_spmv_csr_f64(const nest_desc* desc, int64_t nrows, int
     if (staged) return launch_spmv_staged(p, nrows, ncols, nnz, rowptr, colind, val, x, y, fb, as_stream(stream));
     if (p.x_halo > 0) return launch_spmv_xwin(p, nrows, ncols, rowptr, colind, val, x, y, fb, as_stream(stream));
     return launch_spmv(p, (p.flags & NEST_F_STREAM_HINTS) != 0, nrows, rowptr, colind, val, x, y, fb,
-                       as_stream(stream));
+                       as_stream(stream), nnz);
 }
 
 static size_t align256(size_t b) { return (b + 255) & ~(size_t)255; }
@@ -355,7 +355,7 @@ NEST_API nest_status nest_spmv_csr_f64_hostio(const nest_desc* desc, int64_t nro
     s = staged ? launch_spmv_staged(p, nrows, ncols, nnz, d_rowptr, d_col, d_val, d_x, d_y, fb, st)
         : p.x_halo > 0 ? launch_spmv_xwin(p, nrows, ncols, d_rowptr, d_col, d_val, d_x, d_y, fb, st)
                      : launch_spmv(p, (p.flags & NEST_F_STREAM_HINTS) != 0, nrows, d_rowptr, d_col, d_val,
-                                   d_x, d_y, fb, st);
+                                   d_x, d_y, fb, st, nnz);
     if (s != NEST_OK) return s;
     if ((e = cudaMemcpyAsync(h_y, d_y, (size_t)nrows * 8, cudaMemcpyDeviceToHost, st)))
         return cuda_fail(e, "device->host copy");

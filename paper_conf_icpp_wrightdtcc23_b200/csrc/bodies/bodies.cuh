@@ -50,6 +50,24 @@ struct SpmvBody {
     const double* val;
     const double* x;
     double* y;
+    // L2 prefetch of the team's upcoming nonzeros (blocked schedule): the team
+    // leader prefetches [base + pf_ahead, base + pf_ahead + pf_len) of colind and
+    // val with bulk L2 prefetches (TMA engine), so the groups' loads hit L2.
+    int64_t nnz = 0;
+    int64_t pf_ahead = 0;
+    int64_t pf_len = 0;
+    static constexpr bool kL2Hint = true;
+
+    __device__ __forceinline__ void team_hint(const Loop& L) const {
+        if (pf_len <= 0) return;
+        int64_t b = (L.base + pf_ahead) & ~(int64_t)3;
+        int64_t e = (b + pf_len + 3) & ~(int64_t)3;
+        const int64_t lim = nnz & ~(int64_t)3;
+        if (e > lim) e = lim;
+        if (e <= b) return;
+        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;\n" ::"l"(col + b), "r"((uint32_t)((e - b) * 4)) : "memory");
+        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;\n" ::"l"(val + b), "r"((uint32_t)((e - b) * 8)) : "memory");
+    }
 
     static __device__ __forceinline__ int steps(const SpmvBody&) { return 1; }
     static __device__ __forceinline__ void team_begin(TeamShared&) {}

@@ -63,7 +63,7 @@ int32_t probe_payload(int32_t U);
 // Kernel launchers (one translation unit per body).
 nest_status launch_spmv(const Plan& p, bool hints, int64_t nrows, const int64_t* rowptr,
                         const int32_t* col, const double* val, const double* x, double* y,
-                        unsigned char* fb, cudaStream_t st);
+                        unsigned char* fb, cudaStream_t st, int64_t nnz);
 nest_status launch_spmv_xwin(const Plan& p, int64_t nrows, int64_t ncols, const int64_t* rowptr,
                              const int32_t* col, const double* val, const double* x, double* y,
                              unsigned char* fb, cudaStream_t st);
