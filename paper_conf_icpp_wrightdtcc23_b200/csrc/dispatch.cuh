@@ -12,6 +12,19 @@ namespace nest {
 
 template <class Body, int U, int S, int MODE, int OP>
 nest_status launch_one(const Plan& p, const Body& body, unsigned char* fb, cudaStream_t st) {
+    // a team size the instantiation cannot run (registers) is reported before launching
+    static int max_threads = 0;
+    if (max_threads == 0) {
+        cudaFuncAttributes fa;
+        if (cudaFuncGetAttributes(&fa, nest_kernel<S, MODE, OP, U, Body>) == cudaSuccess)
+            max_threads = fa.maxThreadsPerBlock;
+        else
+            cudaGetLastError();
+    }
+    if (max_threads > 0 && p.block > max_threads)
+        return fail(NEST_ERR_UNSUPPORTED,
+                    "threads_per_team %d exceeds this variant's limit of %d (registers); use a smaller team or "
+                    "outer_unroll", p.block, max_threads);
     nest_kernel<S, MODE, OP, U, Body><<<p.grid, p.block, p.smem_bytes, st>>>(
         body, p.outer, p.slot_bytes, fb, (p.flags & NEST_F_BLOCKED) ? 1 : 0);
     const cudaError_t e = cudaGetLastError();

@@ -1,0 +1,144 @@
+"""Secondary measurements for SURVEY.md §8(d): the other configs' sweeps.
+
+  cfg3  nested stencil loop, N = 2^20, L in {4..64}: simdlen x mode, GB/s and
+        the generic/SPMD time ratio (the paper's Fig 10 question)
+  cfg4  batched 64x64 fp32 matvec, 500k batches: simdlen x mode x unroll, GB/s
+  g100  CSR SpMV on the 100M-nnz matrix (north_star 70% gate), best variants
+
+CUDA events on the current stream, L2 flushed before each timed launch
+(cfg3 launches are us-scale: 20 back-to-back launches per event pair, no
+flush between them -- stated in the output).  Writes one JSON document.
+"""
+import argparse
+import json
+import os
+import statistics
+import sys
+
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import paper_conf_icpp_wrightdtcc23_b200 as P  # noqa: E402
+from nestgen import recipes as R  # noqa: E402
+
+MODES = ("spmd", "generic_smem", "generic_shfl")
+flush = None
+
+
+def timed(fn, iters=5, reps=1, do_flush=True):
+    ts = []
+    fn()
+    torch.cuda.synchronize()
+    for _ in range(iters):
+        if do_flush:
+            P.l2_flush(flush)
+        e0, e1 = torch.cuda.Event(True), torch.cuda.Event(True)
+        e0.record()
+        for _ in range(reps):
+            fn()
+        e1.record()
+        e1.synchronize()
+        ts.append(e0.elapsed_time(e1) / reps)
+    return statistics.median(ts)
+
+
+def cfg3(out):
+    N = 1 << 20
+    res = []
+    for L in R.STENCIL_LS:
+        inp, coef, w = R.stencil_inputs(N, L)
+        t = [torch.from_numpy(a).cuda() for a in (inp, coef, w)]
+        o = torch.empty(N, dtype=torch.float64, device="cuda")
+        B = 8 * (N * L + 2) + 16 * N + 8 * L
+        for S in (1, 2, 4, 8, 16, 32):
+            for mode in MODES:
+                if S == 1 and mode != "spmd":
+                    continue
+                for blocked in (False, True):
+                    ms = timed(lambda: P.nested_stencil_f64(*t, N, L, o, simdlen=S, mode=mode, blocked=blocked,
+                                                            threads_per_team=256), iters=5, reps=20, do_flush=False)
+                    res.append(dict(L=L, S=S, mode=mode, blocked=blocked, ms=ms, GBs=B / ms / 1e6))
+        print("cfg3 L", L, "done", flush=True)
+    summary = {}
+    for L in R.STENCIL_LS:
+        rows = [r for r in res if r["L"] == L]
+        best = min(rows, key=lambda r: r["ms"])
+        s1 = min((r for r in rows if r["S"] == 1), key=lambda r: r["ms"])
+        ratios = {}
+        for S in (2, 4, 8, 16, 32):
+            sp = min((r["ms"] for r in rows if r["S"] == S and r["mode"] == "spmd"))
+            ratios[S] = {m: min(r["ms"] for r in rows if r["S"] == S and r["mode"] == m) / sp
+                         for m in ("generic_smem", "generic_shfl")}
+        summary[L] = dict(best=best, simdlen1=s1, speedup_vs_simdlen1=s1["ms"] / best["ms"],
+                          generic_over_spmd=ratios)
+    out["cfg3"] = dict(note="N=2^20 outer iterations; 20 back-to-back launches per event pair (no flush)",
+                       results=res, summary=summary)
+
+
+def cfg4(out):
+    Bn = 500_000
+    A, x = R.batched_inputs(Bn)
+    tA, tx = torch.from_numpy(A).cuda(), torch.from_numpy(x).cuda()
+    y = torch.empty(Bn * 64, dtype=torch.float32, device="cuda")
+    Bytes = Bn * (64 * 64 * 4 + 64 * 4 + 64 * 4)
+    res = []
+    for S in (1, 2, 4, 8, 16, 32):
+        for mode in MODES:
+            if S == 1 and mode != "spmd":
+                continue
+            for U in (1, 2, 4):
+                for T in (256, 1024):
+                    try:
+                        ms = timed(lambda: P.batched_matvec_f32(tA, tx, Bn, 64, 64, y, simdlen=S, mode=mode,
+                                                                outer_unroll=U, threads_per_team=T))
+                    except P.NestError as e:
+                        print("skip", S, mode, U, T, e)
+                        continue
+                    res.append(dict(S=S, mode=mode, U=U, T=T, ms=ms, GBs=Bytes / ms / 1e6))
+    best = min(res, key=lambda r: r["ms"])
+    s1 = min((r for r in res if r["S"] == 1), key=lambda r: r["ms"])
+    out["cfg4"] = dict(alg_bytes=Bytes, results=res, best=best, simdlen1=s1,
+                       speedup_vs_simdlen1=s1["ms"] / best["ms"])
+    print("cfg4 done", flush=True)
+
+
+def g100(out):
+    spec = R.G100
+    rp, col, val = R.spmv_matrix(spec)
+    x = R.spmv_x(spec)
+    t = [torch.from_numpy(a).cuda() for a in (rp, col, val, x)]
+    y = torch.empty(spec.nrows, dtype=torch.float64, device="cuda")
+    B = val.size * 12 + (spec.nrows + 1) * 8 + spec.nrows * 8 + spec.ncols * 8
+    res = []
+    for S, mode, U, T, blocked in ((1, "spmd", 1, 256, False), (1, "spmd", 1, 1024, True),
+                                   (2, "spmd", 1, 1024, True), (4, "spmd", 1, 1024, True),
+                                   (2, "generic_smem", 1, 1024, True), (8, "spmd", 1, 1024, True)):
+        ms = timed(lambda: P.spmv_csr_f64(*t, y, simdlen=S, mode=mode, outer_unroll=U, threads_per_team=T,
+                                          blocked=blocked), iters=10)
+        res.append(dict(S=S, mode=mode, U=U, T=T, blocked=blocked, ms=ms, GBs=B / ms / 1e6,
+                        frac_of_8TBs=B / ms / 1e6 / 8000.0))
+    out["g100"] = dict(nnz=int(val.size), alg_bytes=B, results=res, best=min(res, key=lambda r: r["ms"]))
+    print("g100 done", flush=True)
+
+
+def main():
+    global flush
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--out", default="gpurun_out/suite.json")
+    ap.add_argument("--only", default="cfg3,cfg4,g100")
+    a = ap.parse_args()
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
+    out = {}
+    for name in a.only.split(","):
+        globals()[name](out)
+    os.makedirs(os.path.dirname(a.out) or ".", exist_ok=True)
+    with open(a.out, "w") as f:
+        json.dump(out, f, indent=1)
+    for k in ("cfg3", "cfg4", "g100"):
+        if k in out:
+            v = out[k]
+            print(k, json.dumps(v.get("summary", v.get("best")), default=str)[:2000])
+
+
+if __name__ == "__main__":
+    main()
