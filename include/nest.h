@@ -98,7 +98,13 @@ enum {
      * cyclically, so the rows in flight on an SM are neighbours (x stays in
      * L1/L2 for banded matrices).  Implies a persistent grid.  Results are
      * identical (the schedule never changes a row's arithmetic). */
-    NEST_F_BLOCKED = 1u << 3
+    NEST_F_BLOCKED = 1u << 3,
+    /* SpMV only: 128-bit loads.  The simd loop runs over pairs of nonzeros
+     * (one 128-bit val load, one 64-bit colind load per pair), lane l taking
+     * pairs l, l+S, ... of the row ("blocked-cyclic" order: real results
+     * differ from the scalar order by rounding only).  Needs 16-byte aligned
+     * val and 8-byte aligned colind. */
+    NEST_F_VEC128 = 1u << 4
 };
 
 /* The nest descriptor: team, thread and simd extents, mode and reduction.

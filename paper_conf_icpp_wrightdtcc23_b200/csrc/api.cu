@@ -71,7 +71,8 @@ static nest_status validate_desc(const nest_desc* d, int32_t* T, int32_t* sharin
     *U = d->outer_unroll ? d->outer_unroll : 1;
     if (*U != 1 && *U != 2 && *U != 4)
         return fail(NEST_ERR_INVALID_ARG, "outer_unroll %d: need 1, 2 or 4", d->outer_unroll);
-    if (d->flags & ~(uint32_t)(NEST_F_PERSISTENT_GRID | NEST_F_STREAM_HINTS | NEST_F_STAGED | NEST_F_BLOCKED))
+    if (d->flags & ~(uint32_t)(NEST_F_PERSISTENT_GRID | NEST_F_STREAM_HINTS | NEST_F_STAGED | NEST_F_BLOCKED |
+                               NEST_F_VEC128))
         return fail(NEST_ERR_INVALID_ARG, "unknown flags 0x%x", d->flags);
     if (d->reserved[0] || d->reserved[1])
         return fail(NEST_ERR_INVALID_ARG, "reserved fields must be 0");
@@ -100,6 +101,10 @@ static nest_status plan_core(const nest_desc* d, int64_t outer, int32_t K, int32
         return fail(NEST_ERR_INVALID_ARG, "x_halo applies to the CSR SpMV only");
     if ((d->flags & NEST_F_STAGED) && !spmv_window)
         return fail(NEST_ERR_INVALID_ARG, "NEST_F_STAGED applies to the CSR SpMV only");
+    if ((d->flags & NEST_F_VEC128) && !spmv_window)
+        return fail(NEST_ERR_INVALID_ARG, "NEST_F_VEC128 applies to the CSR SpMV only");
+    if ((d->flags & NEST_F_VEC128) && (d->x_halo > 0 || (d->flags & NEST_F_STAGED)))
+        return fail(NEST_ERR_UNSUPPORTED, "NEST_F_VEC128 combines with the cyclic or blocked schedule only");
     if ((d->flags & NEST_F_STAGED) && T < 128)
         return fail(NEST_ERR_INVALID_ARG,
                     "NEST_F_STAGED needs threads_per_team >= 128 (producer, 2 gather and >= 1 consumer warps)");
@@ -127,19 +132,17 @@ static nest_status plan_core(const nest_desc* d, int64_t outer, int32_t K, int32
         q.x_halo = d->x_halo;   // stage sizes and grid: plan_spmv_staged (needs nnz)
         q.grid = d->num_teams;
     } else if (d->x_halo > 0) {
-        // x window (spmv_xwin.cuh): ring of 2^k >= 2R + 2H doubles, R = G*U rows per chunk,
-        // plus a double-buffered rowptr stage; always a persistent block schedule.
+        // x window (spmv_xwin.cuh): ring of XW = 2R + 2H doubles (even), R = G*U rows per
+        // chunk, plus a double-buffered rowptr stage; always a persistent block schedule.
         const int64_t R = (int64_t)q.groups * U;
-        const int64_t need = 2 * R + 2 * (int64_t)d->x_halo;
-        int32_t lg = 4;
-        while (((int64_t)1 << lg) < need) ++lg;
-        const int64_t bytes = ((int64_t)8 << lg) + 2 * (R + 1) * 8 + q.smem_bytes;
+        const int64_t xw = (2 * R + 2 * (int64_t)d->x_halo + 1) & ~(int64_t)1;
+        const int64_t bytes = xw * 8 + 2 * (R + 1) * 8 + q.smem_bytes;
         if (bytes > kMaxDynSmem)
             return fail(NEST_ERR_UNSUPPORTED,
                         "x_halo %d with %lld rows per chunk needs %lld B of shared memory (max %d)",
                         d->x_halo, (long long)R, (long long)bytes, kMaxDynSmem);
         q.x_halo = d->x_halo;
-        q.xw_log2 = lg;
+        q.xw = (int32_t)xw;
         q.smem_bytes = (int32_t)bytes;
         if (d->num_teams > 0) {
             q.grid = d->num_teams;
@@ -301,6 +304,9 @@ NEST_API nest_status nest_spmv_csr_f64(const nest_desc* desc, int64_t nrows, int
         return fail(NEST_ERR_UNSUPPORTED, "NEST_F_STAGED needs 16-byte aligned colind, val and x");
     unsigned char* fb = nullptr;
     if ((s = prepare_fallback(p, &fb)) != NEST_OK) return s;
+    if ((p.flags & NEST_F_VEC128) &&
+        ((reinterpret_cast<uintptr_t>(val) & 15) || (reinterpret_cast<uintptr_t>(colind) & 7)))
+        return fail(NEST_ERR_UNSUPPORTED, "NEST_F_VEC128 needs 16-byte aligned val and 8-byte aligned colind");
     if (staged) return launch_spmv_staged(p, nrows, ncols, nnz, rowptr, colind, val, x, y, fb, as_stream(stream));
     if (p.x_halo > 0) return launch_spmv_xwin(p, nrows, ncols, rowptr, colind, val, x, y, fb, as_stream(stream));
     return launch_spmv(p, (p.flags & NEST_F_STREAM_HINTS) != 0, nrows, rowptr, colind, val, x, y, fb,

@@ -30,7 +30,7 @@ __device__ __forceinline__ double ld_stream(const double* p) { return __ldcs(p);
 // sparse_matvec: outer loop over rows on "teams distribute
 // parallel for", inner loop over the row's nonzeros on "simd".  The product is
 // reduced in-group (R2) instead of the paper's atomic update.
-template <bool HINTS>
+template <bool HINTS, bool PIPE = false>
 struct SpmvBody {
     using Acc = double;
     struct Loop {
@@ -69,6 +69,19 @@ struct SpmvBody {
         asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;\n" ::"l"(val + b), "r"((uint32_t)((e - b) * 8)) : "memory");
     }
 
+    // loop-bound pipeline (engine.cuh): rowptr[i], rowptr[i+1] -> 16 shared bytes
+    static constexpr bool kRowptrPipe = PIPE;
+    __device__ __forceinline__ void pipe_issue(int64_t i, unsigned char* slot) const {
+        const unsigned s0 = (unsigned)__cvta_generic_to_shared(slot);
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(s0), "l"(rowptr + i) : "memory");
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(s0 + 8), "l"(rowptr + i + 1) : "memory");
+    }
+    __device__ __forceinline__ Loop pipe_loop(int64_t i, const unsigned char* slot, Step& st) const {
+        const int64_t* v = reinterpret_cast<const int64_t*>(slot);
+        st.i = i;
+        return Loop{v[1] - v[0], v[0]};
+    }
+
     static __device__ __forceinline__ int steps(const SpmvBody&) { return 1; }
     static __device__ __forceinline__ void team_begin(TeamShared&) {}
     static __device__ __forceinline__ void team_end(const SpmvBody&, TeamShared&) {}
@@ -85,6 +98,71 @@ struct SpmvBody {
         const int32_t c = HINTS ? ld_stream(col + k) : __ldg(col + k);
         const double v = HINTS ? ld_stream(val + k) : __ldg(val + k);
         return Red<OP, double>::accum(acc, v, __ldg(x + c));
+    }
+    __device__ __forceinline__ void epilogue(const Step& st, double total) const { y[st.i] = total; }
+};
+
+// ------------------------------------------------- a8 SpMV, 128-bit loads
+// NEST_F_VEC128: the simd loop runs over PAIRS of nonzeros -- pair P holds
+// entries 2P and 2P+1, read with one 128-bit load of val and one 64-bit load of
+// colind -- and lane l takes the row's pairs l, l+S, ... ("blocked-cyclic",
+// DESIGN.md R1: a fixed order different from Fig 8's, so real results differ
+// from the scalar path by rounding only).  Entries of a boundary pair that
+// belong to a neighbouring row are skipped; the pair that would read past nnz
+// falls back to scalar loads.
+template <bool HINTS>
+struct SpmvPairBody {
+    using Acc = double;
+    static constexpr int kLoopUnroll = 1;   // two nonzeros per iteration already
+    struct Loop {
+        int64_t base;   // rowptr[i]
+        int32_t trip;   // pairs covering the row (the simd loop's TripCount)
+        int32_t len;    // nonzeros in the row
+    };
+    struct Step {
+        int64_t i;
+    };
+    static constexpr bool kPrefetch = false;
+    static constexpr bool kTeamState = false;
+    struct TeamShared {
+        int unused;
+    };
+    const int64_t* rowptr;
+    const int32_t* col;
+    const double* val;
+    const double* x;
+    double* y;
+    int64_t nnz;
+
+    static __device__ __forceinline__ int steps(const SpmvPairBody&) { return 1; }
+    static __device__ __forceinline__ void team_begin(TeamShared&) {}
+    static __device__ __forceinline__ void team_end(const SpmvPairBody&, TeamShared&) {}
+
+    __device__ __forceinline__ Loop prologue(int64_t i, int, Step& st, bool, TeamShared&) const {
+        st.i = i;
+        const int64_t b = __ldg(rowptr + i);
+        const int64_t e = __ldg(rowptr + i + 1);
+        return Loop{b, e > b ? (int32_t)(((e + 1) >> 1) - (b >> 1)) : 0, (int32_t)(e - b)};
+    }
+    template <int OP>
+    __device__ __forceinline__ double accum(const Loop& L, int32_t j, double acc) const {
+        const int64_t b = L.base;
+        const int64_t e = b + L.len;
+        const int64_t k0 = ((b >> 1) + j) << 1;   // first entry of the pair
+        int32_t c0, c1;
+        double v0, v1;
+        if (k0 + 1 < nnz) {
+            const int2 c = HINTS ? __ldcs(reinterpret_cast<const int2*>(col + k0))
+                                 : __ldg(reinterpret_cast<const int2*>(col + k0));
+            const double2 v = HINTS ? __ldcs(reinterpret_cast<const double2*>(val + k0))
+                                    : __ldg(reinterpret_cast<const double2*>(val + k0));
+            c0 = c.x, c1 = c.y, v0 = v.x, v1 = v.y;
+        } else {
+            c0 = __ldg(col + k0), v0 = __ldg(val + k0), c1 = c0, v1 = 0.0;
+        }
+        if (k0 >= b) acc = Red<OP, double>::accum(acc, v0, __ldg(x + c0));
+        if (k0 + 1 < e) acc = Red<OP, double>::accum(acc, v1, __ldg(x + c1));
+        return acc;
     }
     __device__ __forceinline__ void epilogue(const Step& st, double total) const { y[st.i] = total; }
 };

@@ -96,6 +96,7 @@ struct StagedLoop {
 struct SpmvStagedBody {
     using Acc = double;
     using Loop = StagedLoop;
+    static constexpr int kLoopUnroll = 1;   // shared-memory operands: no MLP to gain, less code
     struct Step {
         int64_t i;
     };

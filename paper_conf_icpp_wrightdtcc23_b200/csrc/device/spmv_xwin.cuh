@@ -9,7 +9,7 @@
 // R = G*U rows (group g takes rows r0 + u*G + g).  Before a chunk is computed
 // the team has staged, with cp.async into shared memory,
 //   * rowptr[r0 .. r0+R]                      (double-buffered), and
-//   * x[lo, hi), lo = r0 - H, hi = r0 + R + H (a ring of XW = 2^k doubles),
+//   * x[lo, hi), lo = r0 - H, hi = r0 + R + H (a ring of XW doubles),
 // and it stages the NEXT chunk's rowptr and the newly needed tail of x while
 // the current chunk computes.  A nonzero whose column lies in [lo, hi) reads x
 // from the ring (LDS), any other column reads global memory (__ldg), so the
@@ -44,16 +44,25 @@ struct SpmvXwinBody {
     const double* x;
     double* y;
     const double* ring;
-    int64_t lo, span;   // window [lo, lo + span)
-    uint32_t mask;      // XW - 1
+    int32_t lo;         // window [lo, lo + span)
+    uint32_t span;
+    uint32_t lo_slot;   // ring slot of column lo
+    uint32_t xw;        // ring capacity (doubles)
 
     template <int OP>
     __device__ __forceinline__ double accum(const Loop& L, int64_t j, double acc) const {
         const int64_t k = L.base + j;
         const int32_t c = HINTS ? __ldcs(col + k) : __ldg(col + k);
         const double v = HINTS ? __ldcs(val + k) : __ldg(val + k);
-        const double xv = ((uint64_t)((int64_t)c - lo) < (uint64_t)span) ? ring[(uint32_t)c & mask]
-                                                                         : __ldg(x + c);
+        const uint32_t d = (uint32_t)(c - lo);
+        double xv;
+        if (d < span) {
+            uint32_t sl = d + lo_slot;
+            sl = sl >= xw ? sl - xw : sl;
+            xv = ring[sl];
+        } else {
+            xv = __ldg(x + c);
+        }
         return Red<OP, double>::accum(acc, v, xv);
     }
     __device__ __forceinline__ void epilogue(const Step& st, double total) const { y[st.i] = total; }
@@ -68,18 +77,18 @@ struct XwinArgs {
     int64_t nrows;
     int64_t ncols;
     int32_t halo;
-    int32_t xw_log2;
+    int32_t xw;          // ring capacity in doubles (>= 2R + 2H)
     int32_t slot_bytes;
     unsigned char* gfallback;
 };
 
 template <int S, int MODE, int OP, int U, bool HINTS>
-__global__ void spmv_xwin_kernel(const XwinArgs a) {
+__global__ void __launch_bounds__(1024, 2) spmv_xwin_kernel(const XwinArgs a) {
     using Body = SpmvXwinBody<HINTS>;
     using Loop = typename Body::Loop;
     using Step = typename Body::Step;
     extern __shared__ __align__(16) unsigned char smem[];
-    const uint32_t XW = 1u << a.xw_log2;
+    const uint32_t XW = (uint32_t)a.xw;
     double* ring = reinterpret_cast<double*>(smem);
     const SimdGroup<S> g;
     const int G = (int)(blockDim.x / S);
@@ -94,7 +103,7 @@ __global__ void spmv_xwin_kernel(const XwinArgs a) {
     const int64_t gid = (int64_t)blockIdx.x * G + g.group();
     Slot<Loop, U>* slot = group_slot<MODE, Loop, U>(sharing, a.slot_bytes, a.gfallback, g.group(), gid);
 
-    Body body{a.col, a.val, a.x, a.y, ring, 0, 0, XW - 1u};
+    Body body{a.col, a.val, a.x, a.y, ring, 0, 0, 0, XW};
     auto win_lo = [&](int64_t r0) { return r0 - a.halo > 0 ? r0 - a.halo : (int64_t)0; };
     auto win_hi = [&](int64_t r0) {
         const int64_t h = r0 + R + a.halo;
@@ -105,7 +114,14 @@ __global__ void spmv_xwin_kernel(const XwinArgs a) {
         const int64_t rows = re - r0 < R ? re - r0 : R;
         int64_t* dst = rps + buf * (R + 1);
         for (int t = threadIdx.x; t <= rows; t += blockDim.x) cp_async8(dst + t, a.rowptr + r0 + t);
-        for (int64_t c = xf + threadIdx.x; c < xt; c += blockDim.x) cp_async8(ring + ((uint32_t)c & (XW - 1u)), a.x + c);
+        if (xt > xf) {
+            const uint32_t s0 = (uint32_t)(xf % XW);
+            for (uint32_t t = threadIdx.x; t < (uint32_t)(xt - xf); t += blockDim.x) {
+                uint32_t sl = s0 + t;
+                sl = sl >= XW ? sl - XW : sl;
+                cp_async8(ring + sl, a.x + xf + t);
+            }
+        }
         cp_async_commit();
     };
 
@@ -118,8 +134,10 @@ __global__ void spmv_xwin_kernel(const XwinArgs a) {
             const int64_t rend = r0 + R < re ? r0 + R : re;
             const int64_t hi = win_hi(r0);
             if (rend < re) stage(rend, buf ^ 1, hi, win_hi(rend));       // prefetch the next chunk
-            body.lo = win_lo(r0);
-            body.span = hi > body.lo ? hi - body.lo : 0;
+            const int64_t lo = win_lo(r0);
+            body.lo = (int32_t)lo;
+            body.span = hi > lo ? (uint32_t)(hi - lo) : 0u;
+            body.lo_slot = (uint32_t)(lo % XW);
             const int64_t* rp = rps + buf * (R + 1);
             auto gather = [&](Loop (&L)[U], Step (&st)[U], bool) {
                 int cnt = 0;

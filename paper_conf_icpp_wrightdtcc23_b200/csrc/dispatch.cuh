@@ -25,8 +25,13 @@ nest_status launch_one(const Plan& p, const Body& body, unsigned char* fb, cudaS
         return fail(NEST_ERR_UNSUPPORTED,
                     "threads_per_team %d exceeds this variant's limit of %d (registers); use a smaller team or "
                     "outer_unroll", p.block, max_threads);
+    if (p.smem_bytes > 48 * 1024) {
+        const cudaError_t e = cudaFuncSetAttribute(nest_kernel<S, MODE, OP, U, Body>,
+                                                   cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem_bytes);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(max dynamic smem)");
+    }
     nest_kernel<S, MODE, OP, U, Body><<<p.grid, p.block, p.smem_bytes, st>>>(
-        body, p.outer, p.slot_bytes, fb, (p.flags & NEST_F_BLOCKED) ? 1 : 0);
+        body, p.outer, p.slot_bytes, fb, (p.flags & NEST_F_BLOCKED) ? 1 : 0, p.pipe_off);
     const cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e, "kernel launch");
     return NEST_OK;

@@ -34,6 +34,7 @@ struct Plan {
     int32_t nb = 0;        // stage capacity in nonzeros
     int32_t ns = 0;        // stages in flight
     int32_t rmax = 0;      // rows per chunk at most
+    int32_t pipe_off = -1; // nest_kernel loop-bound pipeline ring offset in dynamic smem (-1 = off)
 };
 
 // Record a thread-local error message and return `s`.

@@ -14,6 +14,10 @@ int32_t spmv_payload(int32_t U) {
     return -1;
 }
 
+nest_status launch_spmv_body(const Plan& p, bool hints, const int64_t* rowptr, const int32_t* col,
+                             const double* val, const double* x, double* y, unsigned char* fb,
+                             cudaStream_t st, int64_t nnz, int64_t ahead, int64_t len);
+
 nest_status launch_spmv(const Plan& p, bool hints, int64_t nrows, const int64_t* rowptr,
                         const int32_t* col, const double* val, const double* x, double* y,
                         unsigned char* fb, cudaStream_t st, int64_t nnz) {
@@ -28,14 +32,42 @@ nest_status launch_spmv(const Plan& p, bool hints, int64_t nrows, const int64_t*
         len = (int64_t)(avg * p.groups * p.unroll) + 4;
         ahead = len * rounds;
     }
-    if (hints) {
-        SpmvBody<true> b{rowptr, col, val, x, y};
-        b.nnz = nnz, b.pf_ahead = ahead, b.pf_len = len;
-        return dispatch(p, b, fb, st);
+    // loop-bound pipeline: 3 rounds x U x 16 B per thread after the sharing space
+    static const int pipe = [] {
+        const char* e = std::getenv("NEST_RP_PIPE");
+        return e ? std::atoi(e) : 0;
+    }();
+    Plan q = p;
+    if (pipe) {
+        q.pipe_off = (p.smem_bytes + 15) & ~15;
+        q.smem_bytes = q.pipe_off + 3 * p.unroll * p.block * 16;
     }
-    SpmvBody<false> b{rowptr, col, val, x, y};
+    return launch_spmv_body(q, hints, rowptr, col, val, x, y, fb, st, nnz, ahead, len);
+}
+
+template <bool HINTS, bool PIPE>
+static nest_status launch_spmv_t(const Plan& p, const int64_t* rowptr, const int32_t* col, const double* val,
+                                 const double* x, double* y, unsigned char* fb, cudaStream_t st, int64_t nnz,
+                                 int64_t ahead, int64_t len) {
+    SpmvBody<HINTS, PIPE> b{rowptr, col, val, x, y};
     b.nnz = nnz, b.pf_ahead = ahead, b.pf_len = len;
     return dispatch(p, b, fb, st);
+}
+
+nest_status launch_spmv_body(const Plan& p, bool hints, const int64_t* rowptr, const int32_t* col,
+                             const double* val, const double* x, double* y, unsigned char* fb,
+                             cudaStream_t st, int64_t nnz, int64_t ahead, int64_t len) {
+    const bool pipe = p.pipe_off >= 0;
+    if (p.flags & NEST_F_VEC128) {
+        if (hints) return dispatch(p, SpmvPairBody<true>{rowptr, col, val, x, y, nnz}, fb, st);
+        return dispatch(p, SpmvPairBody<false>{rowptr, col, val, x, y, nnz}, fb, st);
+    }
+    if (hints) {
+        if (pipe) return launch_spmv_t<true, true>(p, rowptr, col, val, x, y, fb, st, nnz, ahead, len);
+        return launch_spmv_t<true, false>(p, rowptr, col, val, x, y, fb, st, nnz, ahead, len);
+    }
+    if (pipe) return launch_spmv_t<false, true>(p, rowptr, col, val, x, y, fb, st, nnz, ahead, len);
+    return launch_spmv_t<false, false>(p, rowptr, col, val, x, y, fb, st, nnz, ahead, len);
 }
 
 }  // namespace nest

@@ -56,7 +56,7 @@ static nest_status xwin_simdlen(const Plan& p, const XwinArgs& a, cudaStream_t s
 nest_status launch_spmv_xwin(const Plan& p, int64_t nrows, int64_t ncols, const int64_t* rowptr,
                              const int32_t* col, const double* val, const double* x, double* y,
                              unsigned char* fb, cudaStream_t st) {
-    const XwinArgs a{rowptr, col, val, x, y, nrows, ncols, p.x_halo, p.xw_log2, p.slot_bytes, fb};
+    const XwinArgs a{rowptr, col, val, x, y, nrows, ncols, p.x_halo, p.xw, p.slot_bytes, fb};
     switch (p.unroll) {
         case 1: return xwin_simdlen<1>(p, a, st);
         case 2: return xwin_simdlen<2>(p, a, st);

@@ -426,3 +426,37 @@ def test_spmv_blocked(P, banded, S, mode):
     visits = torch.zeros(1, dtype=torch.int64, device="cuda")
     y = host(P.nested_stencil_f64(dev(inp), dev(coef), dev(w), N, L, visits=visits, simdlen=S, mode=mode, blocked=True))
     assert np.array_equal(bits(y), bits(yref)) and int(visits.item()) == N
+
+
+# ------------------------------------------------------------------ a8 SpMV, 128-bit pair loads
+@pytest.mark.parametrize("S", SIMDLENS)
+@pytest.mark.parametrize("mode", MODES)
+def test_spmv_vec128(P, banded, cfg1, S, mode):
+    for data in (banded, cfg1):
+        for values in ("int", "real"):
+            rp, col, val, x, yref, aref = data[values]
+            t = [dev(rp), dev(col), dev(val), dev(x)]
+            for U, T, blocked in ((1, 256, False), (2, 1024, True), (4, 128, False), (1, 1024, True)):
+                y = host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, outer_unroll=U, threads_per_team=T,
+                                        blocked=blocked, vec128=True))
+                if values == "int":
+                    assert np.array_equal(bits(y), bits(yref)), (U, T, blocked)
+                else:
+                    assert_close(y, yref, aref, 1e-12)
+
+
+def test_spmv_vec128_odd_tails(P):
+    # odd nnz (the last pair would read past the arrays), empty and 1-nnz rows
+    for lens in ([1, 0, 3, 2, 5, 0, 1], [7] * 33, [0, 0, 1], [2, 1, 64, 33]):
+        rp, col, val, x = _rows_matrix(lens, 200, 5)
+        yref, _ = oracle.spmv_csr_f64(rp, col, val, x)
+        t = [dev(rp), dev(col), dev(val), dev(x)]
+        for S in SIMDLENS:
+            for mode in MODES:
+                y = host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, vec128=True, sharing_bytes=64))
+                assert np.array_equal(bits(y), bits(yref)), (lens, S, mode)
+    rp, col, val, x = _rows_matrix([3, 4], 50, 6)
+    dval = torch.from_numpy(np.concatenate([[0.0], val])).cuda()[1:]
+    with pytest.raises(P.NestError) as e:
+        P.spmv_csr_f64(dev(rp), dev(col), dval, dev(x), vec128=True)
+    assert e.value.status == 2
