@@ -104,7 +104,10 @@ enum {
      * pairs l, l+S, ... of the row ("blocked-cyclic" order: real results
      * differ from the scalar order by rounding only).  Needs 16-byte aligned
      * val and 8-byte aligned colind. */
-    NEST_F_VEC128 = 1u << 4
+    NEST_F_VEC128 = 1u << 4,
+    /* with NEST_F_VEC128: quads instead of pairs (one 128-bit colind load and
+     * two 128-bit val loads per lane iteration); needs 16-byte aligned colind. */
+    NEST_F_VEC_QUAD = 1u << 5
 };
 
 /* The nest descriptor: team, thread and simd extents, mode and reduction.

@@ -27,6 +27,7 @@ NEST_F_STREAM_HINTS = 1 << 1
 NEST_F_STAGED = 1 << 2
 NEST_F_BLOCKED = 1 << 3
 NEST_F_VEC128 = 1 << 4
+NEST_F_VEC_QUAD = 1 << 5
 
 
 class nest_desc(ctypes.Structure):

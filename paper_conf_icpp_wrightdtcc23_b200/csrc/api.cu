@@ -72,7 +72,7 @@ static nest_status validate_desc(const nest_desc* d, int32_t* T, int32_t* sharin
     if (*U != 1 && *U != 2 && *U != 4)
         return fail(NEST_ERR_INVALID_ARG, "outer_unroll %d: need 1, 2 or 4", d->outer_unroll);
     if (d->flags & ~(uint32_t)(NEST_F_PERSISTENT_GRID | NEST_F_STREAM_HINTS | NEST_F_STAGED | NEST_F_BLOCKED |
-                               NEST_F_VEC128))
+                               NEST_F_VEC128 | NEST_F_VEC_QUAD))
         return fail(NEST_ERR_INVALID_ARG, "unknown flags 0x%x", d->flags);
     if (d->reserved[0] || d->reserved[1])
         return fail(NEST_ERR_INVALID_ARG, "reserved fields must be 0");
@@ -103,6 +103,8 @@ static nest_status plan_core(const nest_desc* d, int64_t outer, int32_t K, int32
         return fail(NEST_ERR_INVALID_ARG, "NEST_F_STAGED applies to the CSR SpMV only");
     if ((d->flags & NEST_F_VEC128) && !spmv_window)
         return fail(NEST_ERR_INVALID_ARG, "NEST_F_VEC128 applies to the CSR SpMV only");
+    if ((d->flags & NEST_F_VEC_QUAD) && !(d->flags & NEST_F_VEC128))
+        return fail(NEST_ERR_INVALID_ARG, "NEST_F_VEC_QUAD needs NEST_F_VEC128");
     if ((d->flags & NEST_F_VEC128) && (d->x_halo > 0 || (d->flags & NEST_F_STAGED)))
         return fail(NEST_ERR_UNSUPPORTED, "NEST_F_VEC128 combines with the cyclic or blocked schedule only");
     if ((d->flags & NEST_F_STAGED) && T < 128)
@@ -305,8 +307,10 @@ NEST_API nest_status nest_spmv_csr_f64(const nest_desc* desc, int64_t nrows, int
     unsigned char* fb = nullptr;
     if ((s = prepare_fallback(p, &fb)) != NEST_OK) return s;
     if ((p.flags & NEST_F_VEC128) &&
-        ((reinterpret_cast<uintptr_t>(val) & 15) || (reinterpret_cast<uintptr_t>(colind) & 7)))
-        return fail(NEST_ERR_UNSUPPORTED, "NEST_F_VEC128 needs 16-byte aligned val and 8-byte aligned colind");
+        ((reinterpret_cast<uintptr_t>(val) & 15) ||
+         (reinterpret_cast<uintptr_t>(colind) & ((p.flags & NEST_F_VEC_QUAD) ? 15 : 7))))
+        return fail(NEST_ERR_UNSUPPORTED, "NEST_F_VEC128 needs 16-byte aligned val and %d-byte aligned colind",
+                    (p.flags & NEST_F_VEC_QUAD) ? 16 : 8);
     if (staged) return launch_spmv_staged(p, nrows, ncols, nnz, rowptr, colind, val, x, y, fb, as_stream(stream));
     if (p.x_halo > 0) return launch_spmv_xwin(p, nrows, ncols, rowptr, colind, val, x, y, fb, as_stream(stream));
     return launch_spmv(p, (p.flags & NEST_F_STREAM_HINTS) != 0, nrows, rowptr, colind, val, x, y, fb,

@@ -103,20 +103,22 @@ struct SpmvBody {
 };
 
 // ------------------------------------------------- a8 SpMV, 128-bit loads
-// NEST_F_VEC128: the simd loop runs over PAIRS of nonzeros -- pair P holds
-// entries 2P and 2P+1, read with one 128-bit load of val and one 64-bit load of
-// colind -- and lane l takes the row's pairs l, l+S, ... ("blocked-cyclic",
-// DESIGN.md R1: a fixed order different from Fig 8's, so real results differ
-// from the scalar path by rounding only).  Entries of a boundary pair that
-// belong to a neighbouring row are skipped; the pair that would read past nnz
-// falls back to scalar loads.
-template <bool HINTS>
-struct SpmvPairBody {
+// NEST_F_VEC128 (V = 2) / NEST_F_VEC128 | NEST_F_VEC_QUAD (V = 4): the simd loop
+// runs over V-tuples of nonzeros -- tuple P holds entries VP .. VP+V-1, read
+// with 128-bit loads (V = 2: one double2 of val + one int2 of colind; V = 4:
+// two double2 + one int4) -- and lane l takes the row's tuples l, l+S, ...
+// ("blocked-cyclic", R1: a fixed order different from Fig 8's, so
+// real results differ from the scalar path by rounding only).  Entries of a
+// boundary tuple that belong to a neighbouring row are skipped; a tuple that
+// would read past nnz falls back to scalar loads.
+template <bool HINTS, int V>
+struct SpmvVecBody {
+    static_assert(V == 2 || V == 4, "tuple width");
     using Acc = double;
-    static constexpr int kLoopUnroll = 1;   // two nonzeros per iteration already
+    static constexpr int kLoopUnroll = 1;   // V nonzeros per iteration already
     struct Loop {
         int64_t base;   // rowptr[i]
-        int32_t trip;   // pairs covering the row (the simd loop's TripCount)
+        int32_t trip;   // tuples covering the row (the simd loop's TripCount)
         int32_t len;    // nonzeros in the row
     };
     struct Step {
@@ -134,34 +136,55 @@ struct SpmvPairBody {
     double* y;
     int64_t nnz;
 
-    static __device__ __forceinline__ int steps(const SpmvPairBody&) { return 1; }
+    static __device__ __forceinline__ int steps(const SpmvVecBody&) { return 1; }
     static __device__ __forceinline__ void team_begin(TeamShared&) {}
-    static __device__ __forceinline__ void team_end(const SpmvPairBody&, TeamShared&) {}
+    static __device__ __forceinline__ void team_end(const SpmvVecBody&, TeamShared&) {}
 
     __device__ __forceinline__ Loop prologue(int64_t i, int, Step& st, bool, TeamShared&) const {
         st.i = i;
         const int64_t b = __ldg(rowptr + i);
         const int64_t e = __ldg(rowptr + i + 1);
-        return Loop{b, e > b ? (int32_t)(((e + 1) >> 1) - (b >> 1)) : 0, (int32_t)(e - b)};
+        constexpr int kLog = V == 2 ? 1 : 2;
+        return Loop{b, e > b ? (int32_t)(((e + V - 1) >> kLog) - (b >> kLog)) : 0, (int32_t)(e - b)};
     }
     template <int OP>
     __device__ __forceinline__ double accum(const Loop& L, int32_t j, double acc) const {
         const int64_t b = L.base;
         const int64_t e = b + L.len;
-        const int64_t k0 = ((b >> 1) + j) << 1;   // first entry of the pair
-        int32_t c0, c1;
-        double v0, v1;
-        if (k0 + 1 < nnz) {
-            const int2 c = HINTS ? __ldcs(reinterpret_cast<const int2*>(col + k0))
-                                 : __ldg(reinterpret_cast<const int2*>(col + k0));
-            const double2 v = HINTS ? __ldcs(reinterpret_cast<const double2*>(val + k0))
-                                    : __ldg(reinterpret_cast<const double2*>(val + k0));
-            c0 = c.x, c1 = c.y, v0 = v.x, v1 = v.y;
+        constexpr int kLog = V == 2 ? 1 : 2;
+        const int64_t k0 = ((b >> kLog) + j) << kLog;   // first entry of the tuple
+        int32_t c[V];
+        double v[V];
+        if (k0 + V <= nnz) {
+            if constexpr (V == 2) {
+                const int2 cc = HINTS ? __ldcs(reinterpret_cast<const int2*>(col + k0))
+                                      : __ldg(reinterpret_cast<const int2*>(col + k0));
+                const double2 vv = HINTS ? __ldcs(reinterpret_cast<const double2*>(val + k0))
+                                         : __ldg(reinterpret_cast<const double2*>(val + k0));
+                c[0] = cc.x, c[1] = cc.y, v[0] = vv.x, v[1] = vv.y;
+            } else {
+                const int4 cc = HINTS ? __ldcs(reinterpret_cast<const int4*>(col + k0))
+                                      : __ldg(reinterpret_cast<const int4*>(col + k0));
+                const double2 v0 = HINTS ? __ldcs(reinterpret_cast<const double2*>(val + k0))
+                                         : __ldg(reinterpret_cast<const double2*>(val + k0));
+                const double2 v1 = HINTS ? __ldcs(reinterpret_cast<const double2*>(val + k0 + 2))
+                                         : __ldg(reinterpret_cast<const double2*>(val + k0 + 2));
+                c[0] = cc.x, c[1] = cc.y, c[2] = cc.z, c[3] = cc.w;
+                v[0] = v0.x, v[1] = v0.y, v[2] = v1.x, v[3] = v1.y;
+            }
+        } else if constexpr (V == 2) {   // the last entry of the arrays
+            c[0] = __ldg(col + k0), v[0] = __ldg(val + k0), c[1] = c[0], v[1] = 0.0;
         } else {
-            c0 = __ldg(col + k0), v0 = __ldg(val + k0), c1 = c0, v1 = 0.0;
+#pragma unroll
+            for (int q = 0; q < V; ++q) {
+                const int64_t kq = k0 + q < nnz ? k0 + q : k0;
+                c[q] = __ldg(col + kq);
+                v[q] = __ldg(val + kq);
+            }
         }
-        if (k0 >= b) acc = Red<OP, double>::accum(acc, v0, __ldg(x + c0));
-        if (k0 + 1 < e) acc = Red<OP, double>::accum(acc, v1, __ldg(x + c1));
+#pragma unroll
+        for (int q = 0; q < V; ++q)
+            if (k0 + q >= b && k0 + q < e) acc = Red<OP, double>::accum(acc, v[q], __ldg(x + c[q]));
         return acc;
     }
     __device__ __forceinline__ void epilogue(const Step& st, double total) const { y[st.i] = total; }

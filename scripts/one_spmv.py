@@ -22,6 +22,7 @@ ap.add_argument("--iters", type=int, default=3)
 ap.add_argument("--halo", type=int, default=0)
 ap.add_argument("--staged", type=int, default=0)
 ap.add_argument("--blocked", type=int, default=0)
+ap.add_argument("--vec", type=int, default=0)
 a = ap.parse_args()
 spec = getattr(R, a.spec)
 rp, col, val = R.spmv_matrix(spec)
@@ -32,6 +33,6 @@ flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
 for _ in range(a.iters):
     P.l2_flush(flush)
     P.spmv_csr_f64(*t, y, simdlen=a.S, mode=a.mode, outer_unroll=a.U, stream_hints=bool(a.hints),
-                   threads_per_team=a.T, persistent=bool(a.persistent), x_halo=a.halo, staged=bool(a.staged), blocked=bool(a.blocked))
+                   threads_per_team=a.T, persistent=bool(a.persistent), x_halo=a.halo, staged=bool(a.staged), blocked=bool(a.blocked), vec128=a.vec >= 1, quad=a.vec == 2)
 torch.cuda.synchronize()
 print("done")

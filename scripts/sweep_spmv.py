@@ -52,8 +52,10 @@ def main():
                                               for sg in map(int, a.staged.split(","))
                                               for bl in map(int, a.blocked.split(","))
                                               for vc in map(int, a.vec.split(","))]:
+                        if vc and xh:
+                            continue
                         cfg = dict(simdlen=S, mode=mode, outer_unroll=U, stream_hints=bool(h), threads_per_team=T,
-                                   x_halo=xh, staged=bool(sg), blocked=bool(bl), vec128=bool(vc))
+                                   x_halo=xh, staged=bool(sg), blocked=bool(bl), vec128=vc >= 1, quad=vc == 2)
                         try:
                             P.spmv_csr_f64(*t, y, **cfg)
                         except P.NestError as e:

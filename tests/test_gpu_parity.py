@@ -436,9 +436,10 @@ def test_spmv_vec128(P, banded, cfg1, S, mode):
         for values in ("int", "real"):
             rp, col, val, x, yref, aref = data[values]
             t = [dev(rp), dev(col), dev(val), dev(x)]
-            for U, T, blocked in ((1, 256, False), (2, 1024, True), (4, 128, False), (1, 1024, True)):
+            for U, T, blocked, quad in ((1, 256, False, False), (2, 1024, True, True), (4, 128, False, False),
+                                        (1, 1024, True, False), (1, 512, False, True), (4, 256, True, True)):
                 y = host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, outer_unroll=U, threads_per_team=T,
-                                        blocked=blocked, vec128=True))
+                                        blocked=blocked, vec128=True, quad=quad))
                 if values == "int":
                     assert np.array_equal(bits(y), bits(yref)), (U, T, blocked)
                 else:
@@ -453,8 +454,9 @@ def test_spmv_vec128_odd_tails(P):
         t = [dev(rp), dev(col), dev(val), dev(x)]
         for S in SIMDLENS:
             for mode in MODES:
-                y = host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, vec128=True, sharing_bytes=64))
-                assert np.array_equal(bits(y), bits(yref)), (lens, S, mode)
+                for quad in (False, True):
+                    y = host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, vec128=True, quad=quad, sharing_bytes=64))
+                    assert np.array_equal(bits(y), bits(yref)), (lens, S, mode, quad)
     rp, col, val, x = _rows_matrix([3, 4], 50, 6)
     dval = torch.from_numpy(np.concatenate([[0.0], val])).cuda()[1:]
     with pytest.raises(P.NestError) as e:
