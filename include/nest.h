@@ -99,7 +99,8 @@ enum {
      * L1/L2 for banded matrices).  Implies a persistent grid.  Results are
      * identical (the schedule never changes a row's arithmetic). */
     NEST_F_BLOCKED = 1u << 3,
-    /* SpMV only: 128-bit loads.  The simd loop runs over pairs of nonzeros
+    /* 128-bit loads (SpMV; batched matvec: float4 tuples of a row, needs
+     * n % 4 == 0 and 16-byte aligned A and x).  SpMV: the simd loop runs over pairs of nonzeros
      * (one 128-bit val load, one 64-bit colind load per pair), lane l taking
      * pairs l, l+S, ... of the row ("blocked-cyclic" order: real results
      * differ from the scalar order by rounding only).  Needs 16-byte aligned

@@ -101,8 +101,8 @@ static nest_status plan_core(const nest_desc* d, int64_t outer, int32_t K, int32
         return fail(NEST_ERR_INVALID_ARG, "x_halo applies to the CSR SpMV only");
     if ((d->flags & NEST_F_STAGED) && !spmv_window)
         return fail(NEST_ERR_INVALID_ARG, "NEST_F_STAGED applies to the CSR SpMV only");
-    if ((d->flags & NEST_F_VEC128) && !spmv_window)
-        return fail(NEST_ERR_INVALID_ARG, "NEST_F_VEC128 applies to the CSR SpMV only");
+    if ((d->flags & NEST_F_VEC_QUAD) && !spmv_window)
+        return fail(NEST_ERR_INVALID_ARG, "NEST_F_VEC_QUAD applies to the CSR SpMV only");
     if ((d->flags & NEST_F_VEC_QUAD) && !(d->flags & NEST_F_VEC128))
         return fail(NEST_ERR_INVALID_ARG, "NEST_F_VEC_QUAD needs NEST_F_VEC128");
     if ((d->flags & NEST_F_VEC128) && (d->x_halo > 0 || (d->flags & NEST_F_STAGED)))
@@ -381,6 +381,9 @@ NEST_API nest_status nest_batched_matvec_f32(const nest_desc* desc, int64_t batc
     if (s != NEST_OK) return s;
     if (batch == 0 || m == 0) return NEST_OK;
     if (!y || (n > 0 && (!A || !x))) return fail(NEST_ERR_INVALID_ARG, "A/x/y is NULL");
+    if ((p.flags & NEST_F_VEC128) &&
+        (n % 4 || (reinterpret_cast<uintptr_t>(A) & 15) || (reinterpret_cast<uintptr_t>(x) & 15)))
+        return fail(NEST_ERR_UNSUPPORTED, "NEST_F_VEC128 (batched) needs n %% 4 == 0 and 16-byte aligned A and x");
     unsigned char* fb = nullptr;
     if ((s = prepare_fallback(p, &fb)) != NEST_OK) return s;
     return launch_batched(p, batch, m, n, A, x, y, fb, as_stream(stream));

@@ -229,6 +229,52 @@ struct BatchedBody {
     __device__ __forceinline__ void epilogue(const Step& st, float total) const { y[st.out] = total; }
 };
 
+// NEST_F_VEC128 for the batched body: the simd loop over k runs over float4
+// tuples (lane l takes tuples l, l+S, ...: blocked-cyclic, R1).
+// Requires n % 4 == 0 and 16-byte aligned A and x (checked on the host).
+struct BatchedVecBody {
+    using Acc = float;
+    static constexpr int kLoopUnroll = 1;
+    struct Loop {
+        int64_t base;    // (b*m + r)*n / 4   (float4 index)
+        int64_t xbase;   // b*n / 4
+        int32_t trip;    // n / 4
+        int32_t pad;
+    };
+    struct Step {
+        int64_t out;
+    };
+    static constexpr bool kPrefetch = false;
+    static constexpr bool kTeamState = false;
+    struct TeamShared {
+        int unused;
+    };
+    const float4* A;
+    const float4* x;
+    float* y;
+    int32_t m, n;
+
+    static __device__ __forceinline__ int steps(const BatchedVecBody& b) { return b.m; }
+    static __device__ __forceinline__ void team_begin(TeamShared&) {}
+    static __device__ __forceinline__ void team_end(const BatchedVecBody&, TeamShared&) {}
+
+    __device__ __forceinline__ Loop prologue(int64_t b, int r, Step& st, bool, TeamShared&) const {
+        st.out = b * m + r;
+        const int32_t n4 = n >> 2;
+        return Loop{(b * m + r) * (int64_t)n4, b * (int64_t)n4, n4, 0};
+    }
+    template <int OP>
+    __device__ __forceinline__ float accum(const Loop& L, int32_t j, float acc) const {
+        const float4 a = __ldg(A + L.base + j);
+        const float4 v = __ldg(x + L.xbase + j);
+        acc = Red<OP, float>::accum(acc, a.x, v.x);
+        acc = Red<OP, float>::accum(acc, a.y, v.y);
+        acc = Red<OP, float>::accum(acc, a.z, v.z);
+        return Red<OP, float>::accum(acc, a.w, v.w);
+    }
+    __device__ __forceinline__ void epilogue(const Step& st, float total) const { y[st.out] = total; }
+};
+
 // ---------------------------------------------- a10 nested stencil loop
 // "Benchmark kernel" stand-in with a data-dependent
 // sequential prologue and a non-idempotent side effect

@@ -11,9 +11,13 @@ int32_t batched_payload(int32_t U) {
     }
     return -1;
 }
+static_assert(sizeof(BatchedVecBody::Loop) == sizeof(BatchedBody::Loop), "same generic payload");
 
 nest_status launch_batched(const Plan& p, int64_t, int32_t m, int32_t n, const float* A,
                            const float* x, float* y, unsigned char* fb, cudaStream_t st) {
+    if (p.flags & NEST_F_VEC128)
+        return dispatch(p, BatchedVecBody{reinterpret_cast<const float4*>(A), reinterpret_cast<const float4*>(x), y, m, n},
+                        fb, st);
     return dispatch(p, BatchedBody{A, x, y, m, n}, fb, st);
 }
 

@@ -88,13 +88,15 @@ def cfg4(out):
                 continue
             for U in (1, 2, 4):
                 for T in (256, 1024):
-                    try:
-                        ms = timed(lambda: P.batched_matvec_f32(tA, tx, Bn, 64, 64, y, simdlen=S, mode=mode,
-                                                                outer_unroll=U, threads_per_team=T))
-                    except P.NestError as e:
-                        print("skip", S, mode, U, T, e)
-                        continue
-                    res.append(dict(S=S, mode=mode, U=U, T=T, ms=ms, GBs=Bytes / ms / 1e6))
+                    for vec in (False, True):
+                        try:
+                            ms = timed(lambda: P.batched_matvec_f32(tA, tx, Bn, 64, 64, y, simdlen=S, mode=mode,
+                                                                    outer_unroll=U, threads_per_team=T,
+                                                                    vec128=vec))
+                        except P.NestError as e:
+                            print("skip", S, mode, U, T, vec, str(e)[:80])
+                            continue
+                        res.append(dict(S=S, mode=mode, U=U, T=T, vec128=vec, ms=ms, GBs=Bytes / ms / 1e6))
     best = min(res, key=lambda r: r["ms"])
     s1 = min((r for r in res if r["S"] == 1), key=lambda r: r["ms"])
     out["cfg4"] = dict(alg_bytes=Bytes, results=res, best=best, simdlen1=s1,

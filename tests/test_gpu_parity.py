@@ -462,3 +462,19 @@ def test_spmv_vec128_odd_tails(P):
     with pytest.raises(P.NestError) as e:
         P.spmv_csr_f64(dev(rp), dev(col), dval, dev(x), vec128=True)
     assert e.value.status == 2
+
+
+@pytest.mark.parametrize("S", SIMDLENS)
+@pytest.mark.parametrize("mode", MODES)
+def test_batched_vec128(P, batched, S, mode):
+    for values in ("int", "real"):
+        B, A, x, yref, aref = batched[values]
+        for U, T, blocked in ((1, 256, False), (2, 1024, True), (4, 128, False)):
+            y = host(P.batched_matvec_f32(dev(A), dev(x), B, simdlen=S, mode=mode, outer_unroll=U,
+                                          threads_per_team=T, blocked=blocked, vec128=True))
+            if values == "int":
+                assert np.array_equal(bits(y), bits(yref))
+            else:
+                assert_close(y, yref, aref, 1e-5)
+    with pytest.raises(P.NestError):
+        P.batched_matvec_f32(dev(A[: 3 * 64 * 62].copy()), dev(x[: 3 * 62].copy()), 3, 64, 62, vec128=True)
