@@ -111,18 +111,20 @@ struct SpmvBody {
 // real results differ from the scalar path by rounding only).  Entries of a
 // boundary tuple that belong to a neighbouring row are skipped; a tuple that
 // would read past nnz falls back to scalar loads.
-template <bool HINTS, int V>
+template <bool HINTS, int V, class I = int64_t>
 struct SpmvVecBody {
     static_assert(V == 2 || V == 4, "tuple width");
+    // I: index type of rows and nonzeros (int32_t when nnz and nrows < 2^31:
+    // fewer registers, so two teams of 1024 fit an SM)
     using Acc = double;
     static constexpr int kLoopUnroll = 1;   // V nonzeros per iteration already
     struct Loop {
-        int64_t base;   // rowptr[i]
+        I base;         // rowptr[i]
         int32_t trip;   // tuples covering the row (the simd loop's TripCount)
         int32_t len;    // nonzeros in the row
     };
     struct Step {
-        int64_t i;
+        I i;
     };
     static constexpr bool kPrefetch = false;
     static constexpr bool kTeamState = false;
@@ -141,21 +143,21 @@ struct SpmvVecBody {
     static __device__ __forceinline__ void team_end(const SpmvVecBody&, TeamShared&) {}
 
     __device__ __forceinline__ Loop prologue(int64_t i, int, Step& st, bool, TeamShared&) const {
-        st.i = i;
-        const int64_t b = __ldg(rowptr + i);
-        const int64_t e = __ldg(rowptr + i + 1);
+        st.i = (I)i;
+        const I b = (I)__ldg(rowptr + i);
+        const I e = (I)__ldg(rowptr + i + 1);
         constexpr int kLog = V == 2 ? 1 : 2;
         return Loop{b, e > b ? (int32_t)(((e + V - 1) >> kLog) - (b >> kLog)) : 0, (int32_t)(e - b)};
     }
     template <int OP>
     __device__ __forceinline__ double accum(const Loop& L, int32_t j, double acc) const {
-        const int64_t b = L.base;
-        const int64_t e = b + L.len;
+        const I b = L.base;
+        const I e = b + L.len;
         constexpr int kLog = V == 2 ? 1 : 2;
-        const int64_t k0 = ((b >> kLog) + j) << kLog;   // first entry of the tuple
+        const I k0 = ((b >> kLog) + j) << kLog;   // first entry of the tuple
         int32_t c[V];
         double v[V];
-        if (k0 + V <= nnz) {
+        if ((int64_t)k0 + V <= nnz) {
             if constexpr (V == 2) {
                 const int2 cc = HINTS ? __ldcs(reinterpret_cast<const int2*>(col + k0))
                                       : __ldg(reinterpret_cast<const int2*>(col + k0));
@@ -177,7 +179,7 @@ struct SpmvVecBody {
         } else {
 #pragma unroll
             for (int q = 0; q < V; ++q) {
-                const int64_t kq = k0 + q < nnz ? k0 + q : k0;
+                const I kq = (int64_t)k0 + q < nnz ? k0 + q : k0;
                 c[q] = __ldg(col + kq);
                 v[q] = __ldg(val + kq);
             }

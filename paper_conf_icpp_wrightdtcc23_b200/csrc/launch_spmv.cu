@@ -59,8 +59,14 @@ nest_status launch_spmv_body(const Plan& p, bool hints, const int64_t* rowptr, c
                              cudaStream_t st, int64_t nnz, int64_t ahead, int64_t len) {
     const bool pipe = p.pipe_off >= 0;
     if (p.flags & NEST_F_VEC128) {
-        if (p.flags & NEST_F_VEC_QUAD) return dispatch(p, SpmvVecBody<false, 4>{rowptr, col, val, x, y, nnz}, fb, st);
-        return dispatch(p, SpmvVecBody<false, 2>{rowptr, col, val, x, y, nnz}, fb, st);
+        // 32-bit row / nonzero indices when they fit (fewer registers)
+        const bool i32 = nnz < ((int64_t)1 << 31) - 8 && p.outer < ((int64_t)1 << 31) - 8;
+        if (p.flags & NEST_F_VEC_QUAD) {
+            if (i32) return dispatch(p, SpmvVecBody<false, 4, int32_t>{rowptr, col, val, x, y, nnz}, fb, st);
+            return dispatch(p, SpmvVecBody<false, 4, int64_t>{rowptr, col, val, x, y, nnz}, fb, st);
+        }
+        if (i32) return dispatch(p, SpmvVecBody<false, 2, int32_t>{rowptr, col, val, x, y, nnz}, fb, st);
+        return dispatch(p, SpmvVecBody<false, 2, int64_t>{rowptr, col, val, x, y, nnz}, fb, st);
     }
     if (hints) {
         if (pipe) return launch_spmv_t<true, true>(p, rowptr, col, val, x, y, fb, st, nnz, ahead, len);
