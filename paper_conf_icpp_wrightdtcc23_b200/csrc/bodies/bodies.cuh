@@ -30,15 +30,16 @@ __device__ __forceinline__ double ld_stream(const double* p) { return __ldcs(p);
 // sparse_matvec: outer loop over rows on "teams distribute
 // parallel for", inner loop over the row's nonzeros on "simd".  The product is
 // reduced in-group (R2) instead of the paper's atomic update.
-template <bool HINTS, bool PIPE = false>
+template <bool HINTS, bool PIPE = false, class I = int64_t>
 struct SpmvBody {
     using Acc = double;
+    // I: index type of rows and nonzeros (int32_t when they fit: fewer registers)
     struct Loop {
-        int64_t trip;   // nonzeros in the row (TripCount)
-        int64_t base;   // rowptr[i]
+        I trip;   // nonzeros in the row (TripCount)
+        I base;   // rowptr[i]
     };
     struct Step {
-        int64_t i;
+        I i;
     };
     static constexpr bool kPrefetch = false;  // software-pipelined prologue (costs registers: occupancy)
     static constexpr bool kTeamState = false;
@@ -78,8 +79,8 @@ struct SpmvBody {
     }
     __device__ __forceinline__ Loop pipe_loop(int64_t i, const unsigned char* slot, Step& st) const {
         const int64_t* v = reinterpret_cast<const int64_t*>(slot);
-        st.i = i;
-        return Loop{v[1] - v[0], v[0]};
+        st.i = (I)i;
+        return Loop{(I)(v[1] - v[0]), (I)v[0]};
     }
 
     static __device__ __forceinline__ int steps(const SpmvBody&) { return 1; }
@@ -87,14 +88,14 @@ struct SpmvBody {
     static __device__ __forceinline__ void team_end(const SpmvBody&, TeamShared&) {}
 
     __device__ __forceinline__ Loop prologue(int64_t i, int, Step& st, bool, TeamShared&) const {
-        st.i = i;
-        const int64_t b = __ldg(rowptr + i);
-        const int64_t e = __ldg(rowptr + i + 1);
+        st.i = (I)i;
+        const I b = (I)__ldg(rowptr + i);
+        const I e = (I)__ldg(rowptr + i + 1);
         return Loop{e - b, b};
     }
     template <int OP>
-    __device__ __forceinline__ double accum(const Loop& L, int64_t j, double acc) const {
-        const int64_t k = L.base + j;
+    __device__ __forceinline__ double accum(const Loop& L, I j, double acc) const {
+        const I k = L.base + j;
         const int32_t c = HINTS ? ld_stream(col + k) : __ldg(col + k);
         const double v = HINTS ? ld_stream(val + k) : __ldg(val + k);
         return Red<OP, double>::accum(acc, v, __ldg(x + c));

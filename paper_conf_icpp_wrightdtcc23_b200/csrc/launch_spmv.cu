@@ -1,15 +1,15 @@
 // launch_spmv.cu -- a8 CSR SpMV instantiations.
 #include <cstdlib>
 
-#include "dispatch.cuh"
+#include "spmv_variants.h"
 
 namespace nest {
 
 int32_t spmv_payload(int32_t U) {
     switch (U) {
-        case 1: return payload_bytes<SpmvBody<false>, 1>();
-        case 2: return payload_bytes<SpmvBody<false>, 2>();
-        case 4: return payload_bytes<SpmvBody<false>, 4>();
+        case 1: return payload_bytes<SpmvBody<false, false, int64_t>, 1>();
+        case 2: return payload_bytes<SpmvBody<false, false, int64_t>, 2>();
+        case 4: return payload_bytes<SpmvBody<false, false, int64_t>, 4>();
     }
     return -1;
 }
@@ -49,9 +49,15 @@ template <bool HINTS, bool PIPE>
 static nest_status launch_spmv_t(const Plan& p, const int64_t* rowptr, const int32_t* col, const double* val,
                                  const double* x, double* y, unsigned char* fb, cudaStream_t st, int64_t nnz,
                                  int64_t ahead, int64_t len) {
-    SpmvBody<HINTS, PIPE> b{rowptr, col, val, x, y};
+    // 32-bit row / nonzero indices when they fit (fewer registers)
+    if (nnz < ((int64_t)1 << 31) - 8 && p.outer < ((int64_t)1 << 31) - 8) {
+        SpmvBody<HINTS, PIPE, int32_t> b{rowptr, col, val, x, y};
+        b.nnz = nnz, b.pf_ahead = ahead, b.pf_len = len;
+        return spmv_dispatch(p, b, fb, st);
+    }
+    SpmvBody<HINTS, PIPE, int64_t> b{rowptr, col, val, x, y};
     b.nnz = nnz, b.pf_ahead = ahead, b.pf_len = len;
-    return dispatch(p, b, fb, st);
+    return spmv_dispatch(p, b, fb, st);
 }
 
 nest_status launch_spmv_body(const Plan& p, bool hints, const int64_t* rowptr, const int32_t* col,
@@ -62,11 +68,11 @@ nest_status launch_spmv_body(const Plan& p, bool hints, const int64_t* rowptr, c
         // 32-bit row / nonzero indices when they fit (fewer registers)
         const bool i32 = nnz < ((int64_t)1 << 31) - 8 && p.outer < ((int64_t)1 << 31) - 8;
         if (p.flags & NEST_F_VEC_QUAD) {
-            if (i32) return dispatch(p, SpmvVecBody<false, 4, int32_t>{rowptr, col, val, x, y, nnz}, fb, st);
-            return dispatch(p, SpmvVecBody<false, 4, int64_t>{rowptr, col, val, x, y, nnz}, fb, st);
+            if (i32) return spmv_dispatch(p, SpmvVecBody<false, 4, int32_t>{rowptr, col, val, x, y, nnz}, fb, st);
+            return spmv_dispatch(p, SpmvVecBody<false, 4, int64_t>{rowptr, col, val, x, y, nnz}, fb, st);
         }
-        if (i32) return dispatch(p, SpmvVecBody<false, 2, int32_t>{rowptr, col, val, x, y, nnz}, fb, st);
-        return dispatch(p, SpmvVecBody<false, 2, int64_t>{rowptr, col, val, x, y, nnz}, fb, st);
+        if (i32) return spmv_dispatch(p, SpmvVecBody<false, 2, int32_t>{rowptr, col, val, x, y, nnz}, fb, st);
+        return spmv_dispatch(p, SpmvVecBody<false, 2, int64_t>{rowptr, col, val, x, y, nnz}, fb, st);
     }
     if (hints) {
         if (pipe) return launch_spmv_t<true, true>(p, rowptr, col, val, x, y, fb, st, nnz, ahead, len);

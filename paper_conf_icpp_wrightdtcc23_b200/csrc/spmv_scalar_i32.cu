@@ -1,0 +1,15 @@
+// spmv_scalar_i32.cu -- SpMV instantiations: scalar loads, 32-bit indices.
+#include "dispatch.cuh"
+#include "spmv_variants.h"
+
+namespace nest {
+
+template <class Body>
+nest_status spmv_dispatch(const Plan& p, const Body& body, unsigned char* fb, cudaStream_t st) {
+    return dispatch(p, body, fb, st);
+}
+
+template nest_status spmv_dispatch<SpmvBody<false, false, int32_t>>(const Plan&, const SpmvBody<false, false, int32_t>&, unsigned char*, cudaStream_t);
+template nest_status spmv_dispatch<SpmvBody<true, false, int32_t>>(const Plan&, const SpmvBody<true, false, int32_t>&, unsigned char*, cudaStream_t);
+
+}  // namespace nest
