@@ -82,8 +82,9 @@ enum {
      * loop ("teams distribute" with a persistent league).  Implied when the
      * sharing space falls back to global memory. */
     NEST_F_PERSISTENT_GRID = 1u << 0,
-    /* stream the CSR arrays with L2 evict-first / L1 no-allocate hints and
-     * keep x cached (SpMV only; results unchanged). */
+    /* SpMV cache hints (results unchanged): scalar path -- stream the CSR arrays
+     * with L1 no-allocate / L2 evict-first loads; 128-bit path -- L2 policies:
+     * the CSR arrays evict-first, the x gathers evict-last. */
     NEST_F_STREAM_HINTS = 1u << 1,
     /* SpMV only: warp-specialised pipeline.  Warp 0 of each team stages the
      * team's row chunks (rowptr, colind, val and, with x_halo > 0, the x

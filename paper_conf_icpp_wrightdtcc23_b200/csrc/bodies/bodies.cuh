@@ -26,6 +26,41 @@ namespace nest {
 __device__ __forceinline__ int32_t ld_stream(const int32_t* p) { return __ldcs(p); }
 __device__ __forceinline__ double ld_stream(const double* p) { return __ldcs(p); }
 
+// L2 cache-policy loads (L1 behaviour unchanged): the streamed matrix is
+// evict-first, the gathered x evict-last, so x stays in L2 while the matrix
+// streams through it.
+__device__ __forceinline__ uint64_t l2_policy_evict_first() {
+    uint64_t p;
+    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint64_t l2_policy_evict_last() {
+    uint64_t p;
+    asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ int2 ld_pol(const int2* a, uint64_t pol) {
+    int2 r;
+    asm volatile("ld.global.nc.L2::cache_hint.v2.s32 {%0, %1}, [%2], %3;" : "=r"(r.x), "=r"(r.y) : "l"(a), "l"(pol));
+    return r;
+}
+__device__ __forceinline__ int4 ld_pol(const int4* a, uint64_t pol) {
+    int4 r;
+    asm volatile("ld.global.nc.L2::cache_hint.v4.s32 {%0, %1, %2, %3}, [%4], %5;"
+                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(a), "l"(pol));
+    return r;
+}
+__device__ __forceinline__ double2 ld_pol(const double2* a, uint64_t pol) {
+    double2 r;
+    asm volatile("ld.global.nc.L2::cache_hint.v2.f64 {%0, %1}, [%2], %3;" : "=d"(r.x), "=d"(r.y) : "l"(a), "l"(pol));
+    return r;
+}
+__device__ __forceinline__ double ld_pol(const double* a, uint64_t pol) {
+    double r;
+    asm volatile("ld.global.nc.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(r) : "l"(a), "l"(pol));
+    return r;
+}
+
 // ---------------------------------------------------------------- a8 SpMV
 // sparse_matvec: outer loop over rows on "teams distribute
 // parallel for", inner loop over the row's nonzeros on "simd".  The product is
@@ -160,17 +195,17 @@ struct SpmvVecBody {
         double v[V];
         if ((int64_t)k0 + V <= nnz) {
             if constexpr (V == 2) {
-                const int2 cc = HINTS ? __ldcs(reinterpret_cast<const int2*>(col + k0))
+                const int2 cc = HINTS ? ld_pol(reinterpret_cast<const int2*>(col + k0), l2_policy_evict_first())
                                       : __ldg(reinterpret_cast<const int2*>(col + k0));
-                const double2 vv = HINTS ? __ldcs(reinterpret_cast<const double2*>(val + k0))
+                const double2 vv = HINTS ? ld_pol(reinterpret_cast<const double2*>(val + k0), l2_policy_evict_first())
                                          : __ldg(reinterpret_cast<const double2*>(val + k0));
                 c[0] = cc.x, c[1] = cc.y, v[0] = vv.x, v[1] = vv.y;
             } else {
-                const int4 cc = HINTS ? __ldcs(reinterpret_cast<const int4*>(col + k0))
+                const int4 cc = HINTS ? ld_pol(reinterpret_cast<const int4*>(col + k0), l2_policy_evict_first())
                                       : __ldg(reinterpret_cast<const int4*>(col + k0));
-                const double2 v0 = HINTS ? __ldcs(reinterpret_cast<const double2*>(val + k0))
+                const double2 v0 = HINTS ? ld_pol(reinterpret_cast<const double2*>(val + k0), l2_policy_evict_first())
                                          : __ldg(reinterpret_cast<const double2*>(val + k0));
-                const double2 v1 = HINTS ? __ldcs(reinterpret_cast<const double2*>(val + k0 + 2))
+                const double2 v1 = HINTS ? ld_pol(reinterpret_cast<const double2*>(val + k0 + 2), l2_policy_evict_first())
                                          : __ldg(reinterpret_cast<const double2*>(val + k0 + 2));
                 c[0] = cc.x, c[1] = cc.y, c[2] = cc.z, c[3] = cc.w;
                 v[0] = v0.x, v[1] = v0.y, v[2] = v1.x, v[3] = v1.y;
@@ -187,7 +222,8 @@ struct SpmvVecBody {
         }
 #pragma unroll
         for (int q = 0; q < V; ++q)
-            if (k0 + q >= b && k0 + q < e) acc = Red<OP, double>::accum(acc, v[q], __ldg(x + c[q]));
+            if (k0 + q >= b && k0 + q < e)
+                acc = Red<OP, double>::accum(acc, v[q], HINTS ? ld_pol(x + c[q], l2_policy_evict_last()) : __ldg(x + c[q]));
         return acc;
     }
     __device__ __forceinline__ void epilogue(const Step& st, double total) const { y[st.i] = total; }

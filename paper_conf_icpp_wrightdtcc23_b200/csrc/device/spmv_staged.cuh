@@ -272,11 +272,12 @@ __global__ void __launch_bounds__(1024, 1) spmv_staged_kernel(const StagedArgs a
             if (n4 < 0) n4 = 0;
             int64_t staged_end = cb + n4;
             if (ce4 > cmax && e > cmax && e - cb <= a.nb) {
-                const int64_t tk = cmax + lane;
-                if (lane < 3 && tk < e) {
-                    reinterpret_cast<int32_t*>(st + lay.col_off)[tk - cb] = __ldg(a.col + tk);
-                    reinterpret_cast<double*>(st)[tk - cb] = __ldg(a.val + tk);
-                }
+                // by the arriving lane itself, so its release covers these stores
+                if (lane == 0)
+                    for (int64_t tk = cmax; tk < e; ++tk) {
+                        reinterpret_cast<int32_t*>(st + lay.col_off)[tk - cb] = __ldg(a.col + tk);
+                        reinterpret_cast<double*>(st)[tk - cb] = __ldg(a.val + tk);
+                    }
                 staged_end = e;
             }
             // rowptr[r0 .. r0+rows]: even-length bulk part, the rest by hand
@@ -296,8 +297,8 @@ __global__ void __launch_bounds__(1024, 1) spmv_staged_kernel(const StagedArgs a
                 xa2 = (xa + 1) & ~(int64_t)1;
                 xb2 = xb & ~(int64_t)1;
                 if (xb2 < xa2) xb2 = xa2;
-                if (lane == 1 && (xa & 1) && xa < xb) ring[(uint32_t)(xa % a.xw)] = __ldg(a.x + xa);
-                if (lane == 2 && (xb & 1) && xb - 1 >= xa) ring[(uint32_t)((xb - 1) % a.xw)] = __ldg(a.x + xb - 1);
+                if (lane == 0 && (xa & 1) && xa < xb) ring[(uint32_t)(xa % a.xw)] = __ldg(a.x + xa);
+                if (lane == 0 && (xb & 1) && xb - 1 >= xa) ring[(uint32_t)((xb - 1) % a.xw)] = __ldg(a.x + xb - 1);
             }
             if (lane == 0) {
                 hdr->r0 = r0;

@@ -71,6 +71,7 @@ nest_status launch_spmv_body(const Plan& p, bool hints, const int64_t* rowptr, c
             if (i32) return spmv_dispatch(p, SpmvVecBody<false, 4, int32_t>{rowptr, col, val, x, y, nnz}, fb, st);
             return spmv_dispatch(p, SpmvVecBody<false, 4, int64_t>{rowptr, col, val, x, y, nnz}, fb, st);
         }
+        if (hints && i32) return spmv_dispatch(p, SpmvVecBody<true, 2, int32_t>{rowptr, col, val, x, y, nnz}, fb, st);
         if (i32) return spmv_dispatch(p, SpmvVecBody<false, 2, int32_t>{rowptr, col, val, x, y, nnz}, fb, st);
         return spmv_dispatch(p, SpmvVecBody<false, 2, int64_t>{rowptr, col, val, x, y, nnz}, fb, st);
     }

@@ -1,0 +1,27 @@
+"""compute-sanitizer driver workload: small cfg1-sized SpMV / stencil / batched /
+probe launches in every mode (generic modes exercise the slot handshake and the
+warp barriers).  Run under compute-sanitizer --tool {memcheck,racecheck,synccheck}."""
+import os
+import sys
+
+import numpy as np
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import paper_conf_icpp_wrightdtcc23_b200 as P  # noqa: E402
+from nestgen import recipes as R  # noqa: E402
+
+rp, col, val, x = [torch.from_numpy(a).cuda() for a in R.spmv_inputs(R.CFG1)]
+inp, coef, w = [torch.from_numpy(a).cuda() for a in R.stencil_inputs(4099, 8)]
+A, xb = [torch.from_numpy(a).cuda() for a in R.batched_inputs(64)]
+for S in (2, 8, 32):
+    for mode in ("spmd", "generic_smem", "generic_shfl"):
+        for extra in ({}, {"blocked": True}, {"vec128": True}, {"sharing_bytes": 64}):
+            P.spmv_csr_f64(rp, col, val, x, simdlen=S, mode=mode, **extra)
+        P.spmv_csr_f64(rp, col, val, x, simdlen=S, mode=mode, staged=True, x_halo=100, threads_per_team=256)
+        P.spmv_csr_f64(rp, col, val, x, simdlen=S, mode=mode, x_halo=100)
+        P.nested_stencil_f64(inp, coef, w, 4099, 8, simdlen=S, mode=mode)
+        P.batched_matvec_f32(A, xb, 64, simdlen=S, mode=mode, outer_unroll=2)
+        P.probe_mapping(2, 37, simdlen=S, mode=mode)
+torch.cuda.synchronize()
+print("sanitize workload done")
