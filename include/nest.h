@@ -83,8 +83,8 @@ enum {
      * sharing space falls back to global memory. */
     NEST_F_PERSISTENT_GRID = 1u << 0,
     /* SpMV cache hints (results unchanged): scalar path -- stream the CSR arrays
-     * with L1 no-allocate / L2 evict-first loads; 128-bit path -- L2 policies:
-     * the CSR arrays evict-first, the x gathers evict-last. */
+     * with L1 no-allocate / L2 evict-first loads; 128-bit path -- the CSR
+     * tuples with L1 no-allocate loads (L1 kept for the x gathers). */
     NEST_F_STREAM_HINTS = 1u << 1,
     /* SpMV only: warp-specialised pipeline.  Warp 0 of each team stages the
      * team's row chunks (rowptr, colind, val and, with x_halo > 0, the x

@@ -20,6 +20,10 @@
 
 #include "device/engine.cuh"
 
+#ifndef NEST_VEC_UNROLL
+#define NEST_VEC_UNROLL 1
+#endif
+
 namespace nest {
 
 // Streaming loads: L1 no-allocate + L2 evict-first policy (read once).
@@ -53,6 +57,23 @@ __device__ __forceinline__ int4 ld_pol(const int4* a, uint64_t pol) {
 __device__ __forceinline__ double2 ld_pol(const double2* a, uint64_t pol) {
     double2 r;
     asm volatile("ld.global.nc.L2::cache_hint.v2.f64 {%0, %1}, [%2], %3;" : "=d"(r.x), "=d"(r.y) : "l"(a), "l"(pol));
+    return r;
+}
+// L1 no-allocate loads for data read exactly once (keeps L1 for the x gathers)
+__device__ __forceinline__ int2 ld_na(const int2* a) {
+    int2 r;
+    asm volatile("ld.global.nc.L1::no_allocate.v2.s32 {%0, %1}, [%2];" : "=r"(r.x), "=r"(r.y) : "l"(a));
+    return r;
+}
+__device__ __forceinline__ int4 ld_na(const int4* a) {
+    int4 r;
+    asm volatile("ld.global.nc.L1::no_allocate.v4.s32 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(a));
+    return r;
+}
+__device__ __forceinline__ double2 ld_na(const double2* a) {
+    double2 r;
+    asm volatile("ld.global.nc.L1::no_allocate.v2.f64 {%0, %1}, [%2];" : "=d"(r.x), "=d"(r.y) : "l"(a));
     return r;
 }
 __device__ __forceinline__ double ld_pol(const double* a, uint64_t pol) {
@@ -153,7 +174,7 @@ struct SpmvVecBody {
     // I: index type of rows and nonzeros (int32_t when nnz and nrows < 2^31:
     // fewer registers, so two teams of 1024 fit an SM)
     using Acc = double;
-    static constexpr int kLoopUnroll = 1;   // V nonzeros per iteration already
+    static constexpr int kLoopUnroll = NEST_VEC_UNROLL;   // V nonzeros per iteration already
     struct Loop {
         I base;         // rowptr[i]
         int32_t trip;   // tuples covering the row (the simd loop's TripCount)
@@ -195,17 +216,17 @@ struct SpmvVecBody {
         double v[V];
         if ((int64_t)k0 + V <= nnz) {
             if constexpr (V == 2) {
-                const int2 cc = HINTS ? ld_pol(reinterpret_cast<const int2*>(col + k0), l2_policy_evict_first())
+                const int2 cc = HINTS ? ld_na(reinterpret_cast<const int2*>(col + k0))
                                       : __ldg(reinterpret_cast<const int2*>(col + k0));
-                const double2 vv = HINTS ? ld_pol(reinterpret_cast<const double2*>(val + k0), l2_policy_evict_first())
+                const double2 vv = HINTS ? ld_na(reinterpret_cast<const double2*>(val + k0))
                                          : __ldg(reinterpret_cast<const double2*>(val + k0));
                 c[0] = cc.x, c[1] = cc.y, v[0] = vv.x, v[1] = vv.y;
             } else {
-                const int4 cc = HINTS ? ld_pol(reinterpret_cast<const int4*>(col + k0), l2_policy_evict_first())
+                const int4 cc = HINTS ? ld_na(reinterpret_cast<const int4*>(col + k0))
                                       : __ldg(reinterpret_cast<const int4*>(col + k0));
-                const double2 v0 = HINTS ? ld_pol(reinterpret_cast<const double2*>(val + k0), l2_policy_evict_first())
+                const double2 v0 = HINTS ? ld_na(reinterpret_cast<const double2*>(val + k0))
                                          : __ldg(reinterpret_cast<const double2*>(val + k0));
-                const double2 v1 = HINTS ? ld_pol(reinterpret_cast<const double2*>(val + k0 + 2), l2_policy_evict_first())
+                const double2 v1 = HINTS ? ld_na(reinterpret_cast<const double2*>(val + k0 + 2))
                                          : __ldg(reinterpret_cast<const double2*>(val + k0 + 2));
                 c[0] = cc.x, c[1] = cc.y, c[2] = cc.z, c[3] = cc.w;
                 v[0] = v0.x, v[1] = v0.y, v[2] = v1.x, v[3] = v1.y;
@@ -223,7 +244,7 @@ struct SpmvVecBody {
 #pragma unroll
         for (int q = 0; q < V; ++q)
             if (k0 + q >= b && k0 + q < e)
-                acc = Red<OP, double>::accum(acc, v[q], HINTS ? ld_pol(x + c[q], l2_policy_evict_last()) : __ldg(x + c[q]));
+                acc = Red<OP, double>::accum(acc, v[q], __ldg(x + c[q]));
         return acc;
     }
     __device__ __forceinline__ void epilogue(const Step& st, double total) const { y[st.i] = total; }
