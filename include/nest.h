@@ -193,6 +193,17 @@ nest_status nest_nested_stencil_f64(const nest_desc *desc, int64_t nouter, int32
                                     const double *in, const double *coef, const double *w,
                                     double *out, unsigned long long *visits, void *stream);
 
+/* NEXT-2: laplace3d heat-diffusion step (Fig 10 cost study),
+ * a simd loop WITHOUT a reduction.  u, out f64[nz][ny][nx] row-major (x fastest).
+ * For every interior point (1 <= i < nz-1, 1 <= j < ny-1, 1 <= k < nx-1):
+ *   lap = (((((u[i-1][j][k] + u[i+1][j][k]) + u[i][j-1][k]) + u[i][j+1][k])
+ *            + u[i][j][k-1]) + u[i][j][k+1]) - 6*u[i][j][k]
+ *   out[i][j][k] = u[i][j][k] + alpha*lap      (no FMA contraction)
+ * Boundary points of out are not written.  Outer (parallel) unit = a line
+ * (i, j), simd unit = k.  u and out must not alias. */
+nest_status nest_laplace3d_f64(const nest_desc *desc, int64_t nz, int64_t ny, int64_t nx,
+                               double alpha, const double *u, double *out, void *stream);
+
 /* a2/a5/a6 probe.  out_map int32[grid*block*5] (may be NULL): per thread
  * {getSimdGroup, getSimdGroupId, getSimdGroupSize, isSimdGroupLeader, simdmask}
  * (PAPER.md:507-529).  Then one outer iteration per group (outer = grid*G)

@@ -112,5 +112,17 @@ def batched_inputs(batch: int, m: int = 64, n: int = 64, values: str = "real",
     return A, x
 
 
+# NEXT-2 laplace3d: a (nz, ny, nx) fp64 field, U[-1,1) or integers in {-8..8}
+LAPLACE_SHAPE = (256, 256, 256)
+
+
+def laplace_inputs(nz: int, ny: int, nx: int, values: str = "real", cfg_seed: int = seed(7)):
+    from . import vec_f64
+    if values == "int":
+        return vec_f64(cfg_seed, 41, nz * ny * nx, "int", -8, 8)
+    return vec_f64(cfg_seed, 41, nz * ny * nx, "real")
+
+
 __all__ = ["SpmvSpec", "CFG1", "CFG2", "CFG2_UNIFORM", "G100", "CFG5", "spmv_matrix", "spmv_x",
-           "spmv_inputs", "stencil_inputs", "batched_inputs", "STENCIL_LS", "seed"]
+           "spmv_inputs", "stencil_inputs", "batched_inputs", "STENCIL_LS", "seed", "LAPLACE_SHAPE",
+           "laplace_inputs"]

@@ -35,9 +35,10 @@ def lib():
         L.oracle_simd_owner.argtypes = [i64, i32, vp]
         L.oracle_plan_geometry.argtypes = [i32, i32, i32, i32, vp]
         L.oracle_shard_rows.argtypes = [i64, i32, i32, vp]
+        L.oracle_laplace3d_f64.argtypes = [i64, i64, i64, ctypes.c_double, vp, vp]
         for f in (L.oracle_spmv_csr_f64, L.oracle_batched_matvec_f32, L.oracle_nested_stencil_f64,
                   L.oracle_group_map, L.oracle_simd_owner, L.oracle_plan_geometry,
-                  L.oracle_shard_rows):
+                  L.oracle_shard_rows, L.oracle_laplace3d_f64):
             f.restype = ctypes.c_int
         _lib = L
     return _lib
@@ -118,3 +119,13 @@ def shard_rows(n, P, r):
     if lib().oracle_shard_rows(n, P, r, _p(out)):
         raise ValueError("oracle_shard_rows: bad arguments")
     return tuple(int(v) for v in out)
+
+
+def laplace3d_f64(u, nz, ny, nx, alpha, out=None):
+    """NEXT-2: one Jacobi heat step on the interior; boundary of `out` copied from
+    `out` (default: a copy of u)."""
+    u = _c(u, np.float64)
+    o = u.copy() if out is None else _c(out, np.float64).copy()
+    if lib().oracle_laplace3d_f64(nz, ny, nx, float(alpha), _p(u), _p(o)):
+        raise ValueError("oracle_laplace3d_f64: bad arguments")
+    return o

@@ -120,6 +120,31 @@ int oracle_nested_stencil_f64(int64_t nouter, int32_t L, const double *in, const
     return 0;
 }
 
+/* NEXT-2 -- laplace3d heat-diffusion step ("a simple
+ * three-dimensional heat diffusion kernel called laplace3d"; the paper gives no
+ * formula, R19 fixes the 7-point Jacobi step):
+ *   for i in [1,nz-1), j in [1,ny-1), k in [1,nx-1):
+ *     lap = (((((u[i-1][j][k] + u[i+1][j][k]) + u[i][j-1][k]) + u[i][j+1][k])
+ *              + u[i][j][k-1]) + u[i][j][k+1]) - 6*u[i][j][k]
+ *     out[i][j][k] = u[i][j][k] + alpha*lap
+ * Boundary points of out are left untouched. */
+int oracle_laplace3d_f64(int64_t nz, int64_t ny, int64_t nx, double alpha, const double *u, double *out) {
+    if (nz < 0 || ny < 0 || nx < 0) return 1;
+    for (int64_t i = 1; i < nz - 1; ++i)
+        for (int64_t j = 1; j < ny - 1; ++j)
+            for (int64_t k = 1; k < nx - 1; ++k) {
+                const int64_t c = (i * ny + j) * nx + k;
+                double lap = u[c - ny * nx] + u[c + ny * nx];
+                lap = lap + u[c - nx];
+                lap = lap + u[c + nx];
+                lap = lap + u[c - 1];
+                lap = lap + u[c + 1];
+                lap = lap - 6.0 * u[c];
+                out[c] = u[c] + alpha * lap;
+            }
+    return 0;
+}
+
 /* a2 -- SIMD-group partition of a team of T threads into groups of S adjacent
  * threads, queried per thread as in
  * PAPER.md:507-529.  out[t*5 + {0..4}] = {getSimdGroup, getSimdGroupId,

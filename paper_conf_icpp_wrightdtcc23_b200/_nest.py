@@ -62,6 +62,7 @@ SIGNATURES = {
     "nest_batched_matvec_f32": (_st, [_D, _i64, _i32, _i32, _vp, _vp, _vp, _vp]),
     "nest_nested_stencil_f64": (_st, [_D, _i64, _i32, _vp, _vp, _vp, _vp, _vp, _vp]),
     "nest_probe_mapping": (_st, [_D, _vp, _i64, _vp, _vp, _vp, _vp]),
+    "nest_laplace3d_f64": (_st, [_D, _i64, _i64, _i64, ctypes.c_double, _vp, _vp, _vp]),
     "nest_csr_validate": (_st, [_i64, _i64, _i64, _vp, _vp, _vp, _vp]),
     "nest_util_l2_flush": (_st, [_vp, _sz, _vp]),
     "nest_comm_unique_id": (_st, [_vp]),

@@ -159,6 +159,16 @@ def nested_stencil_f64(inp, coef, w, nouter, L, out=None, visits=None, *, stream
     return out
 
 
+def laplace3d_f64(u, out, nz, ny, nx, alpha, *, stream=None, **cfg):
+    """NEXT-2: one Jacobi heat-diffusion step on the interior (non-reducing simd loop)."""
+    torch = _torch()
+    d = make_desc(**cfg)
+    n = nz * ny * nx
+    check(N.nest_laplace3d_f64(ctypes.byref(d), nz, ny, nx, float(alpha), _dev(u, torch.float64, n, "u"),
+                               _dev(out, torch.float64, n, "out"), _stream(stream)), "nest_laplace3d_f64")
+    return out
+
+
 def probe_mapping(num_teams, trip, *, with_map=True, stream=None, **cfg):
     """a2/a5/a6 probe: returns (map[grid*T,5], hits[trip], owner[trip], totals[grid*G])."""
     torch = _torch()

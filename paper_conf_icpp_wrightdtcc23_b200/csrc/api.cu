@@ -404,6 +404,21 @@ NEST_API nest_status nest_nested_stencil_f64(const nest_desc* desc, int64_t nout
     return launch_stencil(p, nouter, L, in, coef, w, out, visits, fb, as_stream(stream));
 }
 
+NEST_API nest_status nest_laplace3d_f64(const nest_desc* desc, int64_t nz, int64_t ny, int64_t nx,
+                                        double alpha, const double* u, double* out, void* stream) {
+    if (nz < 0 || ny < 0 || nx < 0) return fail(NEST_ERR_INVALID_ARG, "negative extent");
+    const int64_t lines = (nz > 2 && ny > 2) ? (nz - 2) * (ny - 2) : 0;
+    Plan p;
+    nest_status s = make_plan(desc, lines, 1, laplace_payload, &p);
+    if (s != NEST_OK) return s;
+    if (lines == 0 || nx <= 2) return NEST_OK;
+    if (!u || !out) return fail(NEST_ERR_INVALID_ARG, "u/out is NULL");
+    if (u == out) return fail(NEST_ERR_INVALID_ARG, "u and out must not alias (Jacobi step)");
+    unsigned char* fb = nullptr;
+    if ((s = prepare_fallback(p, &fb)) != NEST_OK) return s;
+    return launch_laplace(p, nz, ny, nx, alpha, u, out, fb, as_stream(stream));
+}
+
 NEST_API nest_status nest_probe_mapping(const nest_desc* desc, int32_t* out_map, int64_t trip,
                                         int32_t* hits, int32_t* owner, double* totals,
                                         void* stream) {

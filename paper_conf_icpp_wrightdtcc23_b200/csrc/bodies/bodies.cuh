@@ -392,6 +392,62 @@ struct StencilBody {
     }
 };
 
+// ------------------------------------------------ NEXT-2 laplace3d
+// 3-D heat-diffusion step (the Fig 10 cost study):
+// teams distribute + parallel for over the (i, j) lines of the interior, simd
+// over k -- a simd loop WITHOUT a reduction (kReduce = false).  The prologue
+// (line base offset) is the sequential code between the parallel and the simd
+// loop that decides SPMD vs generic.  Each point:
+//   lap = (((((u[z-1] + u[z+1]) + u[y-1]) + u[y+1]) + u[x-1]) + u[x+1]) - 6 u
+//   out = u + alpha * lap
+// with round-to-nearest intrinsics (no contraction), so every mode and simdlen
+// is bit-identical to the oracle.
+struct LaplaceBody {
+    using Acc = double;
+    static constexpr bool kReduce = false;
+    struct Loop {
+        int64_t trip;   // nx - 2
+        int64_t base;   // index of (i, j, 1)
+    };
+    struct Step {
+        int64_t i;
+    };
+    static constexpr bool kPrefetch = false;
+    static constexpr bool kTeamState = false;
+    struct TeamShared {
+        int unused;
+    };
+    const double* u;
+    double* out;
+    int64_t ny, nx;
+    double alpha;
+
+    static __device__ __forceinline__ int steps(const LaplaceBody&) { return 1; }
+    static __device__ __forceinline__ void team_begin(TeamShared&) {}
+    static __device__ __forceinline__ void team_end(const LaplaceBody&, TeamShared&) {}
+
+    __device__ __forceinline__ Loop prologue(int64_t o, int, Step& st, bool, TeamShared&) const {
+        st.i = o;
+        const int64_t i = 1 + o / (ny - 2), j = 1 + o % (ny - 2);
+        return Loop{nx - 2, (i * ny + j) * nx + 1};
+    }
+    __device__ __forceinline__ void apply(const Loop& L, int64_t j) const {
+        const int64_t c = L.base + j;
+        const int64_t sz = ny * nx;
+        double lap = __dadd_rn(__ldg(u + c - sz), __ldg(u + c + sz));
+        lap = __dadd_rn(lap, __ldg(u + c - nx));
+        lap = __dadd_rn(lap, __ldg(u + c + nx));
+        lap = __dadd_rn(lap, __ldg(u + c - 1));
+        lap = __dadd_rn(lap, __ldg(u + c + 1));
+        const double uc = __ldg(u + c);
+        lap = __dsub_rn(lap, __dmul_rn(6.0, uc));
+        out[c] = __dadd_rn(uc, __dmul_rn(alpha, lap));
+    }
+    template <int OP>
+    __device__ __forceinline__ double accum(const Loop&, int64_t, double acc) const { return acc; }
+    __device__ __forceinline__ void epilogue(const Step&, double) const {}
+};
+
 // ---------------------------------------------------------------- probe
 // One outer iteration per group; the simd loop body records coverage (hits),
 // the executing lane (owner, group 0 only) and counts iterations through the

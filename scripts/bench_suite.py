@@ -104,6 +104,28 @@ def cfg4(out):
     print("cfg4 done", flush=True)
 
 
+def laplace(out):
+    nz, ny, nx = R.LAPLACE_SHAPE
+    u = torch.from_numpy(R.laplace_inputs(nz, ny, nx)).cuda()
+    o = u.clone()
+    B = 8 * nz * ny * nx + 8 * (nz - 2) * (ny - 2) * (nx - 2)   # u read once, interior written
+    res = []
+    for S in (1, 2, 4, 8, 16, 32):
+        for mode in MODES:
+            if S == 1 and mode != "spmd":
+                continue
+            for blocked in (False, True):
+                for T in (256, 1024):
+                    ms = timed(lambda: P.laplace3d_f64(u, o, nz, ny, nx, 0.1, simdlen=S, mode=mode, blocked=blocked,
+                                                       threads_per_team=T), iters=7)
+                    res.append(dict(S=S, mode=mode, blocked=blocked, T=T, ms=ms, GBs=B / ms / 1e6))
+    s1 = min((r for r in res if r["S"] == 1), key=lambda r: r["ms"])
+    fig10 = {m: min(r["ms"] for r in res if r["S"] == 32 and r["mode"] == m) / s1["ms"] for m in MODES}
+    out["laplace"] = dict(shape=[nz, ny, nx], alg_bytes=B, results=res, best=min(res, key=lambda r: r["ms"]),
+                          no_simd=s1, fig10_time_over_no_simd_at_S32=fig10)
+    print("laplace done", flush=True)
+
+
 def g100(out):
     spec = R.G100
     rp, col, val = R.spmv_matrix(spec)
@@ -112,12 +134,13 @@ def g100(out):
     y = torch.empty(spec.nrows, dtype=torch.float64, device="cuda")
     B = val.size * 12 + (spec.nrows + 1) * 8 + spec.nrows * 8 + spec.ncols * 8
     res = []
-    for S, mode, U, T, blocked in ((1, "spmd", 1, 256, False), (1, "spmd", 1, 1024, True),
-                                   (2, "spmd", 1, 1024, True), (4, "spmd", 1, 1024, True),
-                                   (2, "generic_smem", 1, 1024, True), (8, "spmd", 1, 1024, True)):
+    for S, mode, U, T, blocked, vec in ((1, "spmd", 1, 256, False, False), (1, "spmd", 1, 1024, True, True),
+                                        (2, "spmd", 1, 1024, True, True), (2, "spmd", 1, 1024, True, False),
+                                        (4, "spmd", 1, 1024, True, True), (2, "generic_smem", 1, 1024, True, True),
+                                        (8, "spmd", 1, 1024, True, False)):
         ms = timed(lambda: P.spmv_csr_f64(*t, y, simdlen=S, mode=mode, outer_unroll=U, threads_per_team=T,
-                                          blocked=blocked), iters=10)
-        res.append(dict(S=S, mode=mode, U=U, T=T, blocked=blocked, ms=ms, GBs=B / ms / 1e6,
+                                          blocked=blocked, vec128=vec), iters=10)
+        res.append(dict(S=S, mode=mode, U=U, T=T, blocked=blocked, vec128=vec, ms=ms, GBs=B / ms / 1e6,
                         frac_of_8TBs=B / ms / 1e6 / 8000.0))
     out["g100"] = dict(nnz=int(val.size), alg_bytes=B, results=res, best=min(res, key=lambda r: r["ms"]))
     print("g100 done", flush=True)
@@ -127,7 +150,7 @@ def main():
     global flush
     ap = argparse.ArgumentParser()
     ap.add_argument("--out", default="gpurun_out/suite.json")
-    ap.add_argument("--only", default="cfg3,cfg4,g100")
+    ap.add_argument("--only", default="cfg3,cfg4,g100,laplace")
     a = ap.parse_args()
     flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
     out = {}
@@ -136,10 +159,12 @@ def main():
     os.makedirs(os.path.dirname(a.out) or ".", exist_ok=True)
     with open(a.out, "w") as f:
         json.dump(out, f, indent=1)
-    for k in ("cfg3", "cfg4", "g100"):
+    for k in ("cfg3", "cfg4", "g100", "laplace"):
         if k in out:
             v = out[k]
             print(k, json.dumps(v.get("summary", v.get("best")), default=str)[:2000])
+            if k == "laplace":
+                print("fig10", v["fig10_time_over_no_simd_at_S32"])
 
 
 if __name__ == "__main__":

@@ -478,3 +478,17 @@ def test_batched_vec128(P, batched, S, mode):
                 assert_close(y, yref, aref, 1e-5)
     with pytest.raises(P.NestError):
         P.batched_matvec_f32(dev(A[: 3 * 64 * 62].copy()), dev(x[: 3 * 62].copy()), 3, 64, 62, vec128=True)
+
+
+# ------------------------------------------------------------------ NEXT-2 laplace3d (no reduction)
+@pytest.mark.parametrize("S", SIMDLENS)
+@pytest.mark.parametrize("mode", MODES)
+def test_laplace3d(P, S, mode):
+    for (nz, ny, nx), values in (((9, 11, 37), "real"), ((5, 34, 66), "int"), ((3, 3, 3), "real"),
+                                 ((2, 5, 5), "real")):
+        u = R.laplace_inputs(nz, ny, nx, values=values)
+        ref = oracle.laplace3d_f64(u, nz, ny, nx, 0.125)
+        for U, blocked in ((1, False), (2, True), (4, False)):
+            out = dev(u.copy())
+            P.laplace3d_f64(dev(u), out, nz, ny, nx, 0.125, simdlen=S, mode=mode, outer_unroll=U, blocked=blocked)
+            assert np.array_equal(bits(host(out)), bits(ref)), (nz, ny, nx, U, blocked)

@@ -116,3 +116,33 @@ def test_stencil_vs_numpy(L):
             ref2 = w * f(t * coef, axis=1)
             ref2[w == 0] = 0.0
             assert np.array_equal(o2, ref2)
+
+
+# ---------------------------------------------------------------- NEXT-2 laplace3d
+def test_laplace_constant_and_linear_fields_are_fixed_points():
+    nz, ny, nx = 7, 6, 9
+    i, j, k = np.meshgrid(np.arange(nz), np.arange(ny), np.arange(nx), indexing="ij")
+    for u in (np.full((nz, ny, nx), 3.0), (2.0 * i - 3.0 * j + 5.0 * k + 1.0)):
+        out = oracle.laplace3d_f64(u.ravel(), nz, ny, nx, 0.25).reshape(nz, ny, nx)
+        assert np.array_equal(out, u)   # the discrete Laplacian of an affine field is 0
+
+
+def test_laplace_quadratic_closed_form_and_boundary():
+    nz, ny, nx = 5, 5, 8
+    i, j, k = np.meshgrid(np.arange(nz), np.arange(ny), np.arange(nx), indexing="ij")
+    u = (k * k + 2 * i * i).astype(np.float64)   # lap = 2 + 4 = 6 everywhere
+    out = oracle.laplace3d_f64(u.ravel(), nz, ny, nx, 0.5).reshape(nz, ny, nx)
+    assert np.array_equal(out[1:-1, 1:-1, 1:-1], u[1:-1, 1:-1, 1:-1] + 3.0)
+    mask = np.ones_like(u, bool)
+    mask[1:-1, 1:-1, 1:-1] = False
+    assert np.array_equal(out[mask], u[mask])     # boundary untouched
+
+
+def test_laplace_vs_numpy_slicing():
+    nz, ny, nx = 9, 11, 13
+    u = R.laplace_inputs(nz, ny, nx).reshape(nz, ny, nx)
+    out = oracle.laplace3d_f64(u.ravel(), nz, ny, nx, 0.1).reshape(nz, ny, nx)
+    c = u[1:-1, 1:-1, 1:-1]
+    lap = (u[:-2, 1:-1, 1:-1] + u[2:, 1:-1, 1:-1] + u[1:-1, :-2, 1:-1] + u[1:-1, 2:, 1:-1]
+           + u[1:-1, 1:-1, :-2] + u[1:-1, 1:-1, 2:]) - 6 * c
+    assert np.array_equal(out[1:-1, 1:-1, 1:-1], c + 0.1 * lap)   # same order, no FMA in numpy
