@@ -70,7 +70,12 @@ typedef enum {
 typedef enum {
     NEST_MODE_SPMD = 0,          /* all lanes run everything; no communication */
     NEST_MODE_GENERIC_SMEM = 1,  /* main posts loop state in the shared sharing space */
-    NEST_MODE_GENERIC_SHFL = 2   /* main broadcasts loop state with warp shuffles */
+    NEST_MODE_GENERIC_SHFL = 2,  /* main broadcasts loop state with warp shuffles */
+    /* NEXT-1, SpMV only: the paper's TWO-level baseline --
+     * teams in generic mode with an extra team-main warp and a block-level
+     * state machine, `parallel for` over a row's nonzeros on the team's
+     * threads_per_team workers; no simd level (simdlen must be 1). */
+    NEST_MODE_TEAMS_GENERIC = 3
 } nest_mode;
 
 /* Reduction of the simd loop (identity +0.0 / -inf / +inf). */

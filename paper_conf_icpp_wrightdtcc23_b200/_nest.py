@@ -20,7 +20,7 @@ lib = ctypes.CDLL(LIB_PATH)
 
 NEST_ABI_VERSION = 1
 NEST_OK, NEST_ERR_INVALID_ARG, NEST_ERR_UNSUPPORTED, NEST_ERR_CUDA, NEST_ERR_NCCL, NEST_ERR_NO_MEMORY = range(6)
-NEST_MODE_SPMD, NEST_MODE_GENERIC_SMEM, NEST_MODE_GENERIC_SHFL = 0, 1, 2
+NEST_MODE_SPMD, NEST_MODE_GENERIC_SMEM, NEST_MODE_GENERIC_SHFL, NEST_MODE_TEAMS_GENERIC = 0, 1, 2, 3
 NEST_REDUCE_SUM, NEST_REDUCE_MAX, NEST_REDUCE_MIN = 0, 1, 2
 NEST_F_PERSISTENT_GRID = 1 << 0
 NEST_F_STREAM_HINTS = 1 << 1

@@ -11,7 +11,7 @@ import ctypes
 from . import _nest as N
 
 MODES = {"spmd": N.NEST_MODE_SPMD, "generic_smem": N.NEST_MODE_GENERIC_SMEM,
-         "generic_shfl": N.NEST_MODE_GENERIC_SHFL}
+         "generic_shfl": N.NEST_MODE_GENERIC_SHFL, "teams_generic": N.NEST_MODE_TEAMS_GENERIC}
 REDUCES = {"sum": N.NEST_REDUCE_SUM, "max": N.NEST_REDUCE_MAX, "min": N.NEST_REDUCE_MIN}
 SIMDLENS = (1, 2, 4, 8, 16, 32)
 

@@ -60,8 +60,12 @@ static nest_status validate_desc(const nest_desc* d, int32_t* T, int32_t* sharin
         return fail(NEST_ERR_INVALID_ARG, "threads_per_team %d: need a multiple of 32 in [32,1024]", *T);
     if (!valid_simdlen(d->simdlen))
         return fail(NEST_ERR_INVALID_ARG, "simdlen %d: need 1, 2, 4, 8, 16 or 32", d->simdlen);
-    if (d->mode < NEST_MODE_SPMD || d->mode > NEST_MODE_GENERIC_SHFL)
+    if (d->mode < NEST_MODE_SPMD || d->mode > NEST_MODE_TEAMS_GENERIC)
         return fail(NEST_ERR_INVALID_ARG, "mode %d", d->mode);
+    if (d->mode == NEST_MODE_TEAMS_GENERIC && d->simdlen != 1)
+        return fail(NEST_ERR_INVALID_ARG, "NEST_MODE_TEAMS_GENERIC is the two-level baseline: simdlen must be 1");
+    if (d->mode == NEST_MODE_TEAMS_GENERIC && *T > 992)
+        return fail(NEST_ERR_INVALID_ARG, "NEST_MODE_TEAMS_GENERIC: threads_per_team (workers) <= 992 (+ the main warp)");
     if (d->reduce < NEST_REDUCE_SUM || d->reduce > NEST_REDUCE_MIN)
         return fail(NEST_ERR_INVALID_ARG, "reduce %d", d->reduce);
     *sharing = d->sharing_bytes ? d->sharing_bytes : kDefaultSharing;
@@ -101,6 +105,8 @@ static nest_status plan_core(const nest_desc* d, int64_t outer, int32_t K, int32
         return fail(NEST_ERR_INVALID_ARG, "x_halo applies to the CSR SpMV only");
     if ((d->flags & NEST_F_STAGED) && !spmv_window)
         return fail(NEST_ERR_INVALID_ARG, "NEST_F_STAGED applies to the CSR SpMV only");
+    if (d->mode == NEST_MODE_TEAMS_GENERIC && !spmv_window)
+        return fail(NEST_ERR_INVALID_ARG, "NEST_MODE_TEAMS_GENERIC applies to the CSR SpMV only");
     if ((d->flags & NEST_F_VEC_QUAD) && !spmv_window)
         return fail(NEST_ERR_INVALID_ARG, "NEST_F_VEC_QUAD applies to the CSR SpMV only");
     if ((d->flags & NEST_F_VEC_QUAD) && !(d->flags & NEST_F_VEC128))
@@ -298,6 +304,16 @@ NEST_API nest_status nest_spmv_csr_f64(const nest_desc* desc, int64_t nrows, int
     if (nrows == 0) return NEST_OK;
     if (!rowptr || !y) return fail(NEST_ERR_INVALID_ARG, "rowptr/y is NULL");
     if (nnz > 0 && (!colind || !val || !x)) return fail(NEST_ERR_INVALID_ARG, "colind/val/x is NULL");
+    if (desc->mode == NEST_MODE_TEAMS_GENERIC) {
+        if (p.flags & (NEST_F_STAGED | NEST_F_VEC128 | NEST_F_BLOCKED) || p.x_halo > 0)
+            return fail(NEST_ERR_UNSUPPORTED, "NEST_MODE_TEAMS_GENERIC takes no SpMV variant flags");
+        if (desc->num_teams <= 0) {
+            int64_t resident = 0;
+            if ((s = resident_blocks(p.block + 32, 0, &resident)) != NEST_OK) return s;
+            p.grid = (int32_t)(nrows < resident ? nrows : resident);
+        }
+        return launch_spmv_teams_generic(p, nrows, rowptr, colind, val, x, y, as_stream(stream));
+    }
     const bool staged = (p.flags & NEST_F_STAGED) != 0;
     if (staged && (s = plan_spmv_staged(&p, nrows, nnz, desc->sharing_bytes ? desc->sharing_bytes : kDefaultSharing)) != NEST_OK)
         return s;
@@ -335,6 +351,8 @@ NEST_API nest_status nest_spmv_csr_f64_hostio(const nest_desc* desc, int64_t nro
     nest_status s = make_plan(desc, nrows, 1, spmv_payload, &p, true);
     if (s != NEST_OK) return s;
     if (nrows == 0) return NEST_OK;
+    if (desc->mode == NEST_MODE_TEAMS_GENERIC)
+        return fail(NEST_ERR_UNSUPPORTED, "nest_spmv_csr_f64_hostio: use nest_spmv_csr_f64 for NEST_MODE_TEAMS_GENERIC");
     const size_t need = nest_spmv_hostio_workspace_bytes(nrows, ncols, nnz);
     if (!d_workspace || workspace_bytes < need)
         return fail(NEST_ERR_INVALID_ARG, "workspace %zu bytes < %zu", workspace_bytes, need);

@@ -80,6 +80,8 @@ nest_status launch_batched(const Plan& p, int64_t batch, int32_t m, int32_t n, c
 nest_status launch_stencil(const Plan& p, int64_t nouter, int32_t L, const double* in,
                            const double* coef, const double* w, double* out,
                            unsigned long long* visits, unsigned char* fb, cudaStream_t st);
+nest_status launch_spmv_teams_generic(const Plan& p, int64_t nrows, const int64_t* rowptr, const int32_t* col,
+                                      const double* val, const double* x, double* y, cudaStream_t st);
 nest_status launch_laplace(const Plan& p, int64_t nz, int64_t ny, int64_t nx, double alpha, const double* u,
                            double* out, unsigned char* fb, cudaStream_t st);
 nest_status launch_probe(const Plan& p, int32_t* out_map, int64_t trip, int32_t* hits,

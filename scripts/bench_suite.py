@@ -146,11 +146,43 @@ def g100(out):
     print("g100 done", flush=True)
 
 
+def teams(out):
+    """NEXT-1: the paper's two-level baseline (teams distribute in generic mode +
+    parallel for) against the three-level path, CFG2 matrix."""
+    spec = R.CFG2
+    rp, col, val = R.spmv_matrix(spec)
+    x = R.spmv_x(spec)
+    t = [torch.from_numpy(a).cuda() for a in (rp, col, val, x)]
+    y = torch.empty(spec.nrows, dtype=torch.float64, device="cuda")
+    B = val.size * 12 + (spec.nrows + 1) * 8 + spec.nrows * 8 + spec.ncols * 8
+    res = []
+    for T in (32, 64, 128, 256):
+        for teams_ in (0, 148 * 4, 148 * 16):
+            try:
+                ms = timed(lambda: P.spmv_csr_f64(*t, y, simdlen=1, mode="teams_generic", threads_per_team=T,
+                                                  num_teams=teams_), iters=5)
+            except P.NestError as e:
+                print("skip", T, teams_, str(e)[:80])
+                continue
+            res.append(dict(level=2, T=T, num_teams=teams_, ms=ms, GBs=B / ms / 1e6))
+    for S, mode, T, blocked, vec in ((1, "spmd", 1024, True, True), (2, "spmd", 1024, True, True),
+                                     (2, "generic_smem", 1024, True, True), (4, "spmd", 1024, True, True),
+                                     (8, "generic_smem", 256, False, False)):
+        ms = timed(lambda: P.spmv_csr_f64(*t, y, simdlen=S, mode=mode, threads_per_team=T, blocked=blocked,
+                                          vec128=vec), iters=10)
+        res.append(dict(level=3, S=S, mode=mode, T=T, blocked=blocked, vec128=vec, ms=ms, GBs=B / ms / 1e6))
+    two = min((r for r in res if r["level"] == 2), key=lambda r: r["ms"])
+    three = min((r for r in res if r["level"] == 3), key=lambda r: r["ms"])
+    out["teams"] = dict(alg_bytes=B, results=res, best_two_level=two, best_three_level=three,
+                        speedup_three_over_two=two["ms"] / three["ms"])
+    print("teams done", flush=True)
+
+
 def main():
     global flush
     ap = argparse.ArgumentParser()
     ap.add_argument("--out", default="gpurun_out/suite.json")
-    ap.add_argument("--only", default="cfg3,cfg4,g100,laplace")
+    ap.add_argument("--only", default="cfg3,cfg4,g100,laplace,teams")
     a = ap.parse_args()
     flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
     out = {}
@@ -159,6 +191,8 @@ def main():
     os.makedirs(os.path.dirname(a.out) or ".", exist_ok=True)
     with open(a.out, "w") as f:
         json.dump(out, f, indent=1)
+    if "teams" in out:
+        print("teams 3-level/2-level speedup", out["teams"]["speedup_three_over_two"], out["teams"]["best_two_level"])
     for k in ("cfg3", "cfg4", "g100", "laplace"):
         if k in out:
             v = out[k]

@@ -101,3 +101,11 @@ def test_shard_rows_matches_oracle():
     for n, Pn in ((0, 1), (7, 8), (1024, 3), (100_000_000, 8)):
         for r in range(Pn):
             assert P.shard_rows(n, Pn, r) == oracle.shard_rows(n, Pn, r)
+
+
+def test_teams_generic_mode_rules():
+    # the two-level teams-generic baseline: SpMV only, simdlen 1
+    with pytest.raises(P.NestError):
+        P.plan(100, 24, simdlen=2, mode="teams_generic")
+    d = P.make_desc(simdlen=1, mode="teams_generic")
+    assert N.nest_batched_matvec_f32(ctypes.byref(d), 1, 64, 64, None, None, None, None) == N.NEST_ERR_INVALID_ARG

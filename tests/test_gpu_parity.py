@@ -492,3 +492,29 @@ def test_laplace3d(P, S, mode):
             out = dev(u.copy())
             P.laplace3d_f64(dev(u), out, nz, ny, nx, 0.125, simdlen=S, mode=mode, outer_unroll=U, blocked=blocked)
             assert np.array_equal(bits(host(out)), bits(ref)), (nz, ny, nx, U, blocked)
+
+
+# ------------------------------------------------------------------ NEXT-1 two-level teams-generic baseline
+def test_spmv_teams_generic_baseline(P, cfg1, banded):
+    for data in (cfg1, banded):
+        for values in ("int", "real"):
+            rp, col, val, x, yref, aref = data[values]
+            t = [dev(rp), dev(col), dev(val), dev(x)]
+            for T, teams in ((32, 0), (64, 0), (256, 0), (32, 7), (992, 0)):
+                y = host(P.spmv_csr_f64(*t, simdlen=1, mode="teams_generic", threads_per_team=T, num_teams=teams))
+                if values == "int":
+                    assert np.array_equal(bits(y), bits(yref)), (T, teams)
+                else:
+                    assert_close(y, yref, aref, 1e-12)
+    rp, col, val, x, _, _ = cfg1["real"]
+    for op in ("max", "min"):
+        yr, _ = oracle.spmv_csr_f64(rp, col, val, x, op=op)
+        y = host(P.spmv_csr_f64(dev(rp), dev(col), dev(val), dev(x), simdlen=1, mode="teams_generic", reduce=op))
+        assert np.array_equal(y, yr)
+    with pytest.raises(P.NestError):
+        P.spmv_csr_f64(dev(rp), dev(col), dev(val), dev(x), simdlen=2, mode="teams_generic")
+    lens = [0, 0, 1, 33, 64, 0, 1000, 7] * 5
+    rp2, col2, val2, x2 = _rows_matrix(lens, 2000, 9)
+    yr2, _ = oracle.spmv_csr_f64(rp2, col2, val2, x2)
+    y2 = host(P.spmv_csr_f64(dev(rp2), dev(col2), dev(val2), dev(x2), simdlen=1, mode="teams_generic"))
+    assert np.array_equal(bits(y2), bits(yr2))
