@@ -133,7 +133,11 @@ typedef struct {
                                  * [row0 - x_halo, row0 + rows + x_halo) around each team's chunk of
                                  * rows (banded matrices); columns outside it read global memory.
                                  * Results are identical; 0 = no staging. */
-    int32_t reserved[2];        /* must be 0 */
+    int32_t team_chunk;         /* with NEST_F_BLOCKED: outer iterations per team chunk, rounded up to
+                                 * a multiple of G; team b takes chunks b, b + grid, b + 2 grid, ...
+                                 * (its groups cyclically inside a chunk), so all teams sweep the
+                                 * outer range together.  0 = one contiguous range per team. */
+    int32_t reserved;           /* must be 0 */
 } nest_desc;
 
 /* Resolved launch geometry (a1). */

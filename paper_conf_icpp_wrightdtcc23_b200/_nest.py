@@ -36,7 +36,7 @@ class nest_desc(ctypes.Structure):
                 ("mode", ctypes.c_int32), ("reduce", ctypes.c_int32),
                 ("sharing_bytes", ctypes.c_int32), ("flags", ctypes.c_uint32),
                 ("outer_unroll", ctypes.c_int32), ("x_halo", ctypes.c_int32),
-                ("reserved", ctypes.c_int32 * 2)]
+                ("team_chunk", ctypes.c_int32), ("reserved", ctypes.c_int32)]
 
 
 class nest_plan_info(ctypes.Structure):

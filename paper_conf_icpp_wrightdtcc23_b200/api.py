@@ -33,7 +33,8 @@ def make_desc(simdlen: int = 8, mode: str | int = "spmd", reduce: str | int = "s
               threads_per_team: int = 256, num_teams: int = 0, sharing_bytes: int = 0,
               outer_unroll: int = 1, persistent: bool = False, stream_hints: bool = False,
               x_halo: int = 0, staged: bool = False, blocked: bool = False,
-              vec128: bool = False, quad: bool = False, flags: int = 0) -> N.nest_desc:
+              vec128: bool = False, quad: bool = False, team_chunk: int = 0,
+              flags: int = 0) -> N.nest_desc:
     d = N.nest_desc()
     d.abi_version = N.NEST_ABI_VERSION
     d.num_teams = num_teams
@@ -44,6 +45,7 @@ def make_desc(simdlen: int = 8, mode: str | int = "spmd", reduce: str | int = "s
     d.sharing_bytes = sharing_bytes
     d.outer_unroll = outer_unroll
     d.x_halo = x_halo
+    d.team_chunk = team_chunk
     d.flags = flags | (N.NEST_F_PERSISTENT_GRID if persistent else 0) | (
         N.NEST_F_STREAM_HINTS if stream_hints else 0) | (N.NEST_F_STAGED if staged else 0) | (
         N.NEST_F_BLOCKED if blocked else 0) | (N.NEST_F_VEC128 if vec128 or quad else 0) | (

@@ -78,8 +78,10 @@ static nest_status validate_desc(const nest_desc* d, int32_t* T, int32_t* sharin
     if (d->flags & ~(uint32_t)(NEST_F_PERSISTENT_GRID | NEST_F_STREAM_HINTS | NEST_F_STAGED | NEST_F_BLOCKED |
                                NEST_F_VEC128 | NEST_F_VEC_QUAD))
         return fail(NEST_ERR_INVALID_ARG, "unknown flags 0x%x", d->flags);
-    if (d->reserved[0] || d->reserved[1])
-        return fail(NEST_ERR_INVALID_ARG, "reserved fields must be 0");
+    if (d->reserved) return fail(NEST_ERR_INVALID_ARG, "reserved fields must be 0");
+    if (d->team_chunk < 0) return fail(NEST_ERR_INVALID_ARG, "team_chunk %d < 0", d->team_chunk);
+    if (d->team_chunk > 0 && !(d->flags & NEST_F_BLOCKED))
+        return fail(NEST_ERR_INVALID_ARG, "team_chunk needs NEST_F_BLOCKED");
     return NEST_OK;
 }
 
@@ -170,6 +172,13 @@ static nest_status plan_core(const nest_desc* d, int64_t outer, int32_t K, int32
     } else {
         if (needed > INT32_MAX) needed = INT32_MAX;
         q.grid = (int32_t)needed;
+    }
+    if ((d->flags & NEST_F_BLOCKED) && q.grid > 0) {
+        // team chunks: the requested size, or one contiguous range per team;
+        // rounded up to a multiple of G so every group starts inside its chunk
+        int64_t c = d->team_chunk > 0 ? d->team_chunk : (outer + q.grid - 1) / q.grid;
+        if (c < 1) c = 1;
+        q.chunk = (c + q.groups - 1) / q.groups * q.groups;
     }
     *p = q;
     return NEST_OK;

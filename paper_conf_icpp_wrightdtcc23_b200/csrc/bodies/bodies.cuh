@@ -97,7 +97,6 @@ struct SpmvBody {
     struct Step {
         I i;
     };
-    static constexpr bool kPrefetch = false;  // software-pipelined prologue (costs registers: occupancy)
     static constexpr bool kTeamState = false;
     struct TeamShared {
         int unused;
@@ -183,7 +182,6 @@ struct SpmvVecBody {
     struct Step {
         I i;
     };
-    static constexpr bool kPrefetch = false;
     static constexpr bool kTeamState = false;
     struct TeamShared {
         int unused;
@@ -264,7 +262,6 @@ struct BatchedBody {
     struct Step {
         int64_t out;     // b*m + r
     };
-    static constexpr bool kPrefetch = false;  // software-pipelined prologue (costs registers: occupancy)
     static constexpr bool kTeamState = false;
     struct TeamShared {
         int unused;
@@ -304,7 +301,6 @@ struct BatchedVecBody {
     struct Step {
         int64_t out;
     };
-    static constexpr bool kPrefetch = false;
     static constexpr bool kTeamState = false;
     struct TeamShared {
         int unused;
@@ -352,7 +348,6 @@ struct StencilBody {
         double scale;
         int64_t skip;
     };
-    static constexpr bool kPrefetch = false;  // the prologue has a side effect (visits)
     static constexpr bool kTeamState = true;
     struct TeamShared {
         unsigned long long visits;
@@ -412,7 +407,6 @@ struct LaplaceBody {
     struct Step {
         int64_t i;
     };
-    static constexpr bool kPrefetch = false;
     static constexpr bool kTeamState = false;
     struct TeamShared {
         int unused;
@@ -461,7 +455,6 @@ struct ProbeBody {
     struct Step {
         int64_t i;
     };
-    static constexpr bool kPrefetch = false;  // software-pipelined prologue (costs registers: occupancy)
     static constexpr bool kTeamState = false;
     struct TeamShared {
         int unused;

@@ -31,7 +31,7 @@ nest_status launch_one(const Plan& p, const Body& body, unsigned char* fb, cudaS
         if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(max dynamic smem)");
     }
     nest_kernel<S, MODE, OP, U, Body><<<p.grid, p.block, p.smem_bytes, st>>>(
-        body, p.outer, p.slot_bytes, fb, (p.flags & NEST_F_BLOCKED) ? 1 : 0, p.pipe_off);
+        body, p.outer, p.slot_bytes, fb, (p.flags & NEST_F_BLOCKED) ? p.chunk : 0, p.pipe_off);
     const cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e, "kernel launch");
     return NEST_OK;

@@ -27,6 +27,7 @@ struct Plan {
     int32_t smem_bytes = 0;
     uint32_t flags = 0;
     int64_t outer = 0;
+    int64_t chunk = 0;     // NEST_F_BLOCKED: outer iterations per team chunk (a multiple of G)
     int32_t x_halo = 0;    // SpMV x window half-width (0 = none)
     int32_t xw_log2 = 0;   // ring of 2^xw_log2 doubles
     // NEST_F_STAGED pipeline (spmv_staged.cuh)

@@ -23,16 +23,23 @@ ap.add_argument("--halo", type=int, default=0)
 ap.add_argument("--staged", type=int, default=0)
 ap.add_argument("--blocked", type=int, default=0)
 ap.add_argument("--vec", type=int, default=0)
+ap.add_argument("--chunk", type=int, default=0)
+ap.add_argument("--far_den", type=int, default=0, help="override the spec's far-column odds (1/far_den)")
 a = ap.parse_args()
 spec = getattr(R, a.spec)
+if a.far_den:
+    import dataclasses
+    spec = dataclasses.replace(spec, name=f"{spec.name}_far{a.far_den}", far_den=a.far_den)
 rp, col, val = R.spmv_matrix(spec)
 x = R.spmv_x(spec)
 t = [torch.from_numpy(v).cuda() for v in (rp, col, val, x)]
 y = torch.empty(spec.nrows, dtype=torch.float64, device="cuda")
 flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
 for _ in range(a.iters):
+    torch.cuda.synchronize()
     P.l2_flush(flush)
     P.spmv_csr_f64(*t, y, simdlen=a.S, mode=a.mode, outer_unroll=a.U, stream_hints=bool(a.hints),
-                   threads_per_team=a.T, persistent=bool(a.persistent), x_halo=a.halo, staged=bool(a.staged), blocked=bool(a.blocked), vec128=a.vec >= 1, quad=a.vec == 2)
+                   threads_per_team=a.T, persistent=bool(a.persistent), x_halo=a.halo, staged=bool(a.staged), blocked=bool(a.blocked), vec128=a.vec >= 1, quad=a.vec == 2,
+                   team_chunk=a.chunk)
 torch.cuda.synchronize()
 print("done")

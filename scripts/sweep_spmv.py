@@ -28,6 +28,8 @@ def main():
     ap.add_argument("--staged", default="0")
     ap.add_argument("--blocked", default="0")
     ap.add_argument("--vec", default="0")
+    ap.add_argument("--chunks", default="0")
+    ap.add_argument("--tag", default="")
     ap.add_argument("--out", default=None)
     a = ap.parse_args()
     spec = getattr(R, a.spec)
@@ -47,15 +49,16 @@ def main():
                 if S == 1 and mode != "spmd":
                     continue
                 for U in map(int, a.unrolls.split(",")):
-                    for h, xh, sg, bl, vc in [(h, xh, sg, bl, vc) for h in map(int, a.hints.split(","))
+                    for h, xh, sg, bl, vc, ck in [(h, xh, sg, bl, vc, ck) for h in map(int, a.hints.split(","))
                                               for xh in map(int, a.halos.split(","))
                                               for sg in map(int, a.staged.split(","))
                                               for bl in map(int, a.blocked.split(","))
-                                              for vc in map(int, a.vec.split(","))]:
+                                              for vc in map(int, a.vec.split(","))
+                                              for ck in map(int, a.chunks.split(","))]:
                         if vc and xh:
                             continue
                         cfg = dict(simdlen=S, mode=mode, outer_unroll=U, stream_hints=bool(h), threads_per_team=T,
-                                   x_halo=xh, staged=bool(sg), blocked=bool(bl), vec128=vc >= 1, quad=vc == 2)
+                                   x_halo=xh, staged=bool(sg), blocked=bool(bl), vec128=vc >= 1, quad=vc == 2, team_chunk=ck if bl else 0)
                         try:
                             P.spmv_csr_f64(*t, y, **cfg)
                         except P.NestError as e:
@@ -73,7 +76,7 @@ def main():
                             e1.synchronize()
                             ts.append(e0.elapsed_time(e1))
                         ms = float(np.median(ts))
-                        r = dict(T=T, S=S, mode=mode, U=U, hints=h, halo=xh, staged=sg, blocked=bl, vec=vc, ms=ms, min_ms=min(ts), GBs=B / ms / 1e6)
+                        r = dict(T=T, S=S, mode=mode, U=U, hints=h, halo=xh, staged=sg, blocked=bl, vec=vc, chunk=ck, tag=a.tag, ms=ms, min_ms=min(ts), GBs=B / ms / 1e6)
                         res.append(r)
                         print(json.dumps(r), flush=True)
     best = min(res, key=lambda r: r["ms"])

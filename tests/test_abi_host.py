@@ -79,7 +79,7 @@ def test_plan_rejects_bad_abi_version_and_reserved():
     info = N.nest_plan_info()
     assert N.nest_plan(ctypes.byref(d), 10, 0, ctypes.byref(info)) == N.NEST_ERR_INVALID_ARG
     d = P.make_desc()
-    d.reserved[1] = 5
+    d.reserved = 5
     assert N.nest_plan(ctypes.byref(d), 10, 0, ctypes.byref(info)) == N.NEST_ERR_INVALID_ARG
     assert b"reserved" in N.nest_last_error()
 
@@ -109,3 +109,15 @@ def test_teams_generic_mode_rules():
         P.plan(100, 24, simdlen=2, mode="teams_generic")
     d = P.make_desc(simdlen=1, mode="teams_generic")
     assert N.nest_batched_matvec_f32(ctypes.byref(d), 1, 64, 64, None, None, None, None) == N.NEST_ERR_INVALID_ARG
+
+
+def test_team_chunk_validation():
+    # team_chunk needs the blocked schedule and is non-negative
+    with pytest.raises(P.NestError) as e:
+        P.plan(1000, 24, team_chunk=64)
+    assert e.value.status == N.NEST_ERR_INVALID_ARG and "NEST_F_BLOCKED" in str(e.value)
+    with pytest.raises(P.NestError) as e:
+        P.plan(1000, 24, team_chunk=-1, blocked=True, num_teams=4)
+    assert e.value.status == N.NEST_ERR_INVALID_ARG
+    info = P.plan(1000, 24, team_chunk=100, blocked=True, num_teams=4)
+    assert info["grid"] == 4

@@ -412,11 +412,16 @@ def test_spmv_blocked(P, banded, S, mode):
     for values in ("int", "real"):
         rp, col, val, x, yref, aref = banded[values]
         t = [dev(rp), dev(col), dev(val), dev(x)]
-        for U, T, teams in ((1, 1024, 0), (2, 256, 0), (4, 512, 7), (1, 64, 1)):
+        y0 = host(P.spmv_csr_f64(*t, simdlen=S, mode=mode))
+        # team_chunk: round-robin team chunks (rounded up to a multiple of G)
+        for U, T, teams, chunk in ((1, 1024, 0, 0), (2, 256, 0, 0), (4, 512, 7, 0), (1, 64, 1, 0),
+                                   (1, 1024, 0, 1), (2, 256, 3, 100), (1, 128, 0, 3000), (4, 64, 5, 64)):
             y = host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, outer_unroll=U, threads_per_team=T,
-                                    num_teams=teams, blocked=True))
+                                    num_teams=teams, blocked=True, team_chunk=chunk))
+            # the schedule never changes a row's arithmetic: bit-identical to the cyclic run
+            assert np.array_equal(bits(y), bits(y0)), (U, T, teams, chunk)
             if values == "int":
-                assert np.array_equal(bits(y), bits(yref)), (U, T, teams)
+                assert np.array_equal(bits(y), bits(yref)), (U, T, teams, chunk)
             else:
                 assert_close(y, yref, aref, 1e-12)
     # stencil and batched under the blocked schedule too (the flag is generic)
@@ -424,8 +429,11 @@ def test_spmv_blocked(P, banded, S, mode):
     inp, coef, w = R.stencil_inputs(N, L, values="int")
     yref, _, _ = oracle.nested_stencil_f64(inp, coef, w, N, L)
     visits = torch.zeros(1, dtype=torch.int64, device="cuda")
-    y = host(P.nested_stencil_f64(dev(inp), dev(coef), dev(w), N, L, visits=visits, simdlen=S, mode=mode, blocked=True))
-    assert np.array_equal(bits(y), bits(yref)) and int(visits.item()) == N
+    for chunk in (0, 37, 1000):
+        visits.zero_()
+        y = host(P.nested_stencil_f64(dev(inp), dev(coef), dev(w), N, L, visits=visits, simdlen=S, mode=mode,
+                                      blocked=True, team_chunk=chunk))
+        assert np.array_equal(bits(y), bits(yref)) and int(visits.item()) == N, chunk
 
 
 # ------------------------------------------------------------------ a8 SpMV, 128-bit pair loads
