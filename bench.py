@@ -334,44 +334,97 @@ def run_gpu(args, rank, world, local_rank):
         print(json.dumps(line), flush=True)
         return
 
-    # ---- N > 1: row-partitioned SpMV, NCCL all-gather of x inside each step
-    comm = P.Comm()
+    # ---- N > 1: row-partitioned SpMV (weak scaling: spec.nrows rows per rank).
+    # Two exchange strategies, both timed: "xpeer" (NEXT-4, the headline) -- x
+    # stays distributed and the SpMV's simd lanes gather remote x from the
+    # owner's slice over NVLink, bracketed by peer-memory barriers -- and
+    # "allgather" (a12) -- NCCL all-gather of x into x_full, then the local SpMV.
+    cfg = cfg_of(HEADLINE)
     xchunk = -(-gspec.ncols // world)
     xb = min(rank * xchunk, gspec.ncols)
     xl = R.spmv_x(gspec, begin=xb, n=min(xchunk, gspec.ncols - xb))
-    d_xl = torch.zeros(xchunk, dtype=torch.float64, device=dev)
-    d_xl[:xl.size] = torch.from_numpy(xl).to(dev)
-    d_xf = torch.empty(xchunk * world, dtype=torch.float64, device=dev)
+    h_xl = torch.zeros(xchunk, dtype=torch.float64).pin_memory()
+    h_xl[:xl.size] = torch.from_numpy(xl)
+    d_xl = h_xl.to(dev)
     d_y = torch.empty(nloc, dtype=torch.float64, device=dev)
-    cfg = dict(simdlen=4, mode="spmd", outer_unroll=1)
-    step = lambda: comm.spmv_csr_f64(gspec.nrows, gspec.ncols, d_rp, d_col, d_val, d_xl, d_xf, d_y, **cfg)
-    for _ in range(args.warmup):
-        step()
-    torch.cuda.synchronize()
-    dist.barrier()
-    with ClockSampler(local_rank) as clk:
-        torch.cuda.synchronize()
-        ts = time_steps(torch, step, flush, P, args.steps)
-        torch.cuda.synchronize()
-    dist.barrier()
-    ms_local = sum(ts) / len(ts)
-    t = torch.tensor([ms_local], dtype=torch.float64, device=dev)
-    dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    ms = float(t.item())
     nnz_t = torch.tensor([nnz], dtype=torch.int64, device=dev)
     dist.all_reduce(nnz_t)
     B = alg_bytes(gspec.nrows, gspec.ncols, int(nnz_t.item()))
+
+    def timed(step, iters):
+        for _ in range(args.warmup):
+            step()
+        torch.cuda.synchronize()
+        dist.barrier()
+        with ClockSampler(local_rank) as clk:
+            torch.cuda.synchronize()
+            ts = time_steps(torch, step, flush, P, iters)
+            torch.cuda.synchronize()
+        dist.barrier()
+        t = torch.tensor([sum(ts) / len(ts)], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)   # max over ranks
+        return float(t.item()), clk.summary()
+
+    res = {}
+    comm = None
+    y_ag = None
+    if not SHARE_GPU:   # NCCL needs one GPU per rank
+        comm = P.Comm()
+        d_xf = torch.empty(xchunk * world, dtype=torch.float64, device=dev)
+        res["allgather"] = timed(lambda: comm.spmv_csr_f64(gspec.nrows, gspec.ncols, d_rp, d_col, d_val, d_xl,
+                                                           d_xf, d_y, **cfg), args.steps)
+        y_ag = d_y.clone()
+    xp_err = None
+    try:
+        xp = P.XPeer(gspec.ncols)
+        xp.set_local_x(d_xl)
+        res["xpeer"] = timed(lambda: xp.spmv_csr_f64(gspec.nrows, d_rp, d_col, d_val, d_y, **cfg), args.steps)
+        # R16: same rows, same variant -> same bits (even nnz offsets)
+        same = bool(torch.equal(d_y, y_ag)) if y_ag is not None else None
+        # e2e through the public API: H2D of the local CSR and x slice from pinned
+        # memory, the peer-gather SpMV, D2H of y_local -- all inside the timed region
+        h_y = torch.empty(nloc, dtype=torch.float64).pin_memory()
+
+        def e2e_step():
+            a = h_rp.to(dev, non_blocking=True)
+            c = h_col.to(dev, non_blocking=True)
+            v = h_val.to(dev, non_blocking=True)
+            xl_d = h_xl.to(dev, non_blocking=True)
+            xp.set_local_x(xl_d)
+            h_y.copy_(xp.spmv_csr_f64(gspec.nrows, a, c, v, **cfg), non_blocking=True)
+        ms_e2e, _ = timed(e2e_step, max(3, args.steps // 20))
+        e2e = {"value": B / (ms_e2e / 1e3) / 1e9, "unit": UNIT, "ms_per_step": ms_e2e,
+               "h2d_bytes_per_step": (h_rp.numel() + h_col.numel() // 2 + h_val.numel() + h_xl.numel()) * 8,
+               "d2h_bytes_per_step": nloc * 8}
+    except P.NestError as e:   # reported, and the all-gather number stands in
+        xp_err, same, e2e = str(e), None, None
+    head = "xpeer" if "xpeer" in res else "allgather"
+    ms, clocks = res[head]
     if rank == 0:
         line = {"metric": METRIC, "value": B / (ms / 1e3) / 1e9, "unit": UNIT, "n_gpus": world,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
                 "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
                 "config": {"workload": f"row-partitioned CSR SpMV fp64, {spec.nrows} rows per rank "
                                        f"(global {gspec.nrows}), nnz/row U{{{spec.nnz_min}..{spec.nnz_max}}}, "
-                                       "NCCL all-gather of x each step", "parallelism": f"rows/{world}",
-                           "l2": "flushed between timed steps", **cfg},
-                "gpu_launches": 2 * args.steps, "clocks": clk.summary(), "e2e": None}
+                                       f"banded+far; x exchange: {head}", "parallelism": f"rows/{world}",
+                           "l2": "flushed between timed steps", "variant": "blocked teams + 128-bit pair loads",
+                           **cfg},
+                "exchange": {k: {"ms_per_step": v[0], "GBs": B / (v[0] / 1e3) / 1e9} for k, v in res.items()},
+                "xpeer_error": xp_err, "xpeer_bitwise_equal_allgather": same,
+                "gpu_launches": args.steps * (3 if head == "xpeer" else 1),
+                "gpu_launches_detail": ("per step: barrier + SpMV + barrier kernels (+ l2_flush outside the events)"
+                                        if head == "xpeer" else "per step: SpMV kernel + NCCL all-gather"),
+                "clocks": clocks, "e2e": e2e}
         print(json.dumps(line), flush=True)
-    comm.close()
+    if "xpeer" in res:
+        xp.close()
+    if comm is not None:
+        comm.close()
+
+
+# Developer check of the N > 1 code path on a one-GPU box: every rank on cuda:0,
+# gloo process group, the NCCL all-gather leg skipped (timings are meaningless).
+SHARE_GPU = os.environ.get("NEST_BENCH_SHARE_GPU") == "1"
 
 
 def main():
@@ -386,10 +439,10 @@ def main():
     args.warmup = max(args.warmup, 3)
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
-    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    local_rank = 0 if SHARE_GPU else int(os.environ.get("LOCAL_RANK", "0"))
     if world > 1:
         import torch.distributed as dist
-        backend = "gloo" if args.impl == "reference" else "nccl"
+        backend = "gloo" if args.impl == "reference" or SHARE_GPU else "nccl"
         if backend == "nccl":
             import torch
             torch.cuda.set_device(local_rank)

@@ -100,10 +100,12 @@ enum {
      * aligned colind, val and x.  Results are identical to the unstaged path. */
     NEST_F_STAGED = 1u << 2,
     /* "teams distribute" with a static block schedule: team b owns the
-     * contiguous outer range [b*C, (b+1)*C) and its SIMD groups take it
-     * cyclically, so the rows in flight on an SM are neighbours (x stays in
-     * L1/L2 for banded matrices).  Implies a persistent grid.  Results are
-     * identical (the schedule never changes a row's arithmetic). */
+     * contiguous outer range [b*C, (b+1)*C) (C = ceil(outer / grid) rounded up
+     * to a multiple of G, or team_chunk: then chunks b, b + grid, ...) and its
+     * SIMD groups take it cyclically, so the rows in flight on an SM are
+     * neighbours (x stays in L1/L2 for banded matrices).  Implies a persistent
+     * grid.  Results are identical (the schedule never changes a row's
+     * arithmetic). */
     NEST_F_BLOCKED = 1u << 3,
     /* 128-bit loads (SpMV; batched matvec: float4 tuples of a row, needs
      * n % 4 == 0 and 16-byte aligned A and x).  SpMV: the simd loop runs over pairs of nonzeros
@@ -256,6 +258,57 @@ nest_status nest_spmv_csr_f64_dist(const nest_desc *desc, nest_comm *comm, int64
                                    const int64_t *rowptr_local, const int32_t *colind,
                                    const double *val, const double *x_local, double *x_full,
                                    double *y_local, void *stream);
+
+/* ---- NEXT-4: comm-free row-partitioned SpMV over peer memory ----
+ * Same row and x partition as nest_spmv_csr_f64_dist, but x is never gathered:
+ * every rank keeps its x slice (xchunk = ceil(ncols_global / nranks) doubles) in
+ * a library-owned buffer that all peers map (CUDA IPC; NVLink/NVSwitch loads),
+ * and the simd lanes of the SpMV read x[c] straight from the owner's slice
+ * (owner = c / xchunk).  Ordering between ranks uses a flag barrier in peer
+ * memory (system-scope release/acquire), no NCCL.  Results are bit-identical to
+ * the single-GPU kernel at the same (simdlen, mode, variant) (R16).
+ *
+ * Set-up (collective over the ranks, in this order):
+ *   nest_xpeer_create(nranks, rank, ncols_global, &xp, handle)  -> this rank's
+ *       handle blob (nest_xpeer_handle_bytes() bytes: IPC handles of its x slice
+ *       and barrier flags);
+ *   the caller all-gathers the blobs (e.g. torch.distributed), rank order;
+ *   nest_xpeer_open(xp, all_blobs)  -> maps every peer's slice and flags.
+ * The current device must be the rank's GPU; peers on other GPUs need P2P
+ * access (NVLink), which nest_xpeer_open enables. */
+typedef struct nest_xpeer nest_xpeer;
+size_t nest_xpeer_handle_bytes(void);
+nest_status nest_xpeer_create(int32_t nranks, int32_t rank, int64_t ncols_global, nest_xpeer **out,
+                              uint8_t *handle /* [nest_xpeer_handle_bytes()] */);
+nest_status nest_xpeer_open(nest_xpeer *xp, const uint8_t *all_handles /* [nranks][handle_bytes] */);
+/* Single-process form (tests, or one process driving several slices): `slices`
+ * is a HOST array of nranks device pointers to the ranks' x slices (xchunk
+ * doubles each, caller-owned, readable from the current device).  No barrier:
+ * the caller orders writes to the slices against the SpMV. */
+nest_status nest_xpeer_create_local(int32_t nranks, int32_t rank, int64_t ncols_global,
+                                    const double *const *slices, nest_xpeer **out);
+/* Device pointer of this rank's x slice (xchunk doubles; the caller writes its
+ * part of x here, entries past ncols_global on the tail rank are never read). */
+double *nest_xpeer_local_x(nest_xpeer *xp);
+int64_t nest_xpeer_xchunk(const nest_xpeer *xp);
+/* Stream-ordered device-to-device copy of min(n, slice length) doubles from
+ * x_local (device) into this rank's slice; slice length = min(xchunk,
+ * ncols_global - rank*xchunk).  IPC form only. */
+nest_status nest_xpeer_set_x(nest_xpeer *xp, const double *x_local, int64_t n, void *stream);
+/* Stream-ordered barrier over the ranks (all prior work of every rank on its
+ * stream, including writes to its x slice, is visible to all peers after it). */
+nest_status nest_xpeer_barrier(nest_xpeer *xp, void *stream);
+/* barrier; y_local = A[local rows] x with peer gathers of x; barrier (so the
+ * caller may overwrite its slice on return).  Arguments as
+ * nest_spmv_csr_f64_dist (GLOBAL column indices, 0-based local rowptr).
+ * Variants: the cyclic / blocked schedules, scalar or 128-bit pair loads
+ * (NEST_F_VEC128 without NEST_F_VEC_QUAD); NEST_F_STAGED, x_halo and
+ * NEST_MODE_TEAMS_GENERIC return NEST_ERR_UNSUPPORTED. */
+nest_status nest_spmv_csr_f64_xpeer(const nest_desc *desc, nest_xpeer *xp, int64_t nrows_global,
+                                    int64_t nrows_local, int64_t nnz_local, const int64_t *rowptr_local,
+                                    const int32_t *colind, const double *val, double *y_local,
+                                    void *stream);
+nest_status nest_xpeer_destroy(nest_xpeer *xp);
 
 /* Release library-owned device scratch of the current device. */
 nest_status nest_shutdown(void);

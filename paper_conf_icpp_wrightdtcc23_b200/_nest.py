@@ -69,6 +69,16 @@ SIGNATURES = {
     "nest_comm_init": (_st, [_vp, _i32, _i32, ctypes.POINTER(_vp)]),
     "nest_comm_destroy": (_st, [_vp]),
     "nest_spmv_csr_f64_dist": (_st, [_D, _vp, _i64, _i64, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _vp]),
+    "nest_xpeer_handle_bytes": (_sz, []),
+    "nest_xpeer_create": (_st, [_i32, _i32, _i64, ctypes.POINTER(_vp), _vp]),
+    "nest_xpeer_open": (_st, [_vp, _vp]),
+    "nest_xpeer_create_local": (_st, [_i32, _i32, _i64, ctypes.POINTER(_vp), ctypes.POINTER(_vp)]),
+    "nest_xpeer_local_x": (_vp, [_vp]),
+    "nest_xpeer_xchunk": (_i64, [_vp]),
+    "nest_xpeer_set_x": (_st, [_vp, _vp, _i64, _vp]),
+    "nest_xpeer_barrier": (_st, [_vp, _vp]),
+    "nest_spmv_csr_f64_xpeer": (_st, [_D, _vp, _i64, _i64, _i64, _vp, _vp, _vp, _vp, _vp]),
+    "nest_xpeer_destroy": (_st, [_vp]),
     "nest_shutdown": (_st, []),
 }
 

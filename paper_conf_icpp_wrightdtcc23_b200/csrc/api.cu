@@ -234,7 +234,7 @@ nest_status fallback_scratch(size_t bytes, unsigned char** out) {
     return NEST_OK;
 }
 
-static nest_status prepare_fallback(const Plan& p, unsigned char** fb) {
+nest_status prepare_fallback(const Plan& p, unsigned char** fb) {
     *fb = nullptr;
     if (!p.fallback) return NEST_OK;
     const size_t bytes = (size_t)p.grid * (size_t)p.groups * (size_t)p.payload_bytes;

@@ -82,11 +82,56 @@ __device__ __forceinline__ double ld_pol(const double* a, uint64_t pol) {
     return r;
 }
 
+// ------------------------------------------------------- x access policies
+// How the SpMV's simd loop reads x[c] (c a global column index).
+// XLocal: x is one array in this GPU's memory (single GPU, or the all-gathered
+// x_full of the row-partitioned SpMV).
+struct XLocal {
+    const double* p;
+    __device__ __forceinline__ double operator()(int32_t c) const { return __ldg(p + c); }
+};
+
+// Unsigned 32-bit division by a run-time constant d >= 1 (round-up multiplier:
+// q = (t + ((n - t) >> 1)) >> (l - 1), t = umulhi(n, m), l = ceil(log2 d)).
+struct FastDivU32 {
+    uint32_t d, m, s;   // s = l (0 when d == 1)
+    static FastDivU32 make(uint32_t d) {
+        FastDivU32 f{d, 0u, 0u};
+        if (d > 1) {
+            uint32_t l = 0;
+            while (l < 32 && (1ull << l) < d) ++l;
+            f.m = (uint32_t)(((1ull << 32) * ((1ull << l) - d)) / d + 1);
+            f.s = l;
+        }
+        return f;
+    }
+    __device__ __forceinline__ uint32_t div(uint32_t n) const {
+        if (s == 0) return n;
+        const uint32_t t = __umulhi(n, m);
+        return (t + ((n - t) >> 1)) >> (s - 1);
+    }
+};
+
+// XPeer (NEXT-4, comm-free row-partitioned SpMV): x stays distributed -- rank
+// o owns columns [o*chunk, (o+1)*chunk) in its own memory -- and the simd loop
+// gathers x[c] straight from the owner's slice through its peer mapping
+// (NVLink loads from the simd lanes; no all-gather).
+struct XPeer {
+    const double* const* slices;   // device array: nranks peer-mapped slice pointers
+    FastDivU32 chunk;
+    __device__ __forceinline__ double operator()(int32_t c) const {
+        const uint32_t o = chunk.div((uint32_t)c);
+        const double* s = reinterpret_cast<const double*>(
+            __ldg(reinterpret_cast<const unsigned long long*>(slices) + o));
+        return __ldg(s + ((uint32_t)c - o * chunk.d));
+    }
+};
+
 // ---------------------------------------------------------------- a8 SpMV
 // sparse_matvec: outer loop over rows on "teams distribute
 // parallel for", inner loop over the row's nonzeros on "simd".  The product is
 // reduced in-group (R2) instead of the paper's atomic update.
-template <bool HINTS, bool PIPE = false, class I = int64_t>
+template <bool HINTS, bool PIPE = false, class I = int64_t, class XA = XLocal>
 struct SpmvBody {
     using Acc = double;
     // I: index type of rows and nonzeros (int32_t when they fit: fewer registers)
@@ -104,7 +149,7 @@ struct SpmvBody {
     const int64_t* rowptr;
     const int32_t* col;
     const double* val;
-    const double* x;
+    XA x;   // x access (XLocal: x[c]; XPeer: the owner rank's slice)
     double* y;
     // L2 prefetch of the team's upcoming nonzeros (blocked schedule): the team
     // leader prefetches [base + pf_ahead, base + pf_ahead + pf_len) of colind and
@@ -153,7 +198,7 @@ struct SpmvBody {
         const I k = L.base + j;
         const int32_t c = HINTS ? ld_stream(col + k) : __ldg(col + k);
         const double v = HINTS ? ld_stream(val + k) : __ldg(val + k);
-        return Red<OP, double>::accum(acc, v, __ldg(x + c));
+        return Red<OP, double>::accum(acc, v, x(c));
     }
     __device__ __forceinline__ void epilogue(const Step& st, double total) const { y[st.i] = total; }
 };
@@ -167,7 +212,7 @@ struct SpmvBody {
 // real results differ from the scalar path by rounding only).  Entries of a
 // boundary tuple that belong to a neighbouring row are skipped; a tuple that
 // would read past nnz falls back to scalar loads.
-template <bool HINTS, int V, class I = int64_t>
+template <bool HINTS, int V, class I = int64_t, class XA = XLocal>
 struct SpmvVecBody {
     static_assert(V == 2 || V == 4, "tuple width");
     // I: index type of rows and nonzeros (int32_t when nnz and nrows < 2^31:
@@ -189,7 +234,7 @@ struct SpmvVecBody {
     const int64_t* rowptr;
     const int32_t* col;
     const double* val;
-    const double* x;
+    XA x;   // x access (XLocal: x[c]; XPeer: the owner rank's slice)
     double* y;
     int64_t nnz;
 
@@ -242,7 +287,7 @@ struct SpmvVecBody {
 #pragma unroll
         for (int q = 0; q < V; ++q)
             if (k0 + q >= b && k0 + q < e)
-                acc = Red<OP, double>::accum(acc, v[q], __ldg(x + c[q]));
+                acc = Red<OP, double>::accum(acc, v[q], x(c[q]));
         return acc;
     }
     __device__ __forceinline__ void epilogue(const Step& st, double total) const { y[st.i] = total; }

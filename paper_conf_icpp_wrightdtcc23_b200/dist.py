@@ -95,3 +95,86 @@ class Comm:
                                        _stream(stream)),
               "nest_spmv_csr_f64_dist")
         return y_local
+
+
+class XPeer:
+    """NEXT-4: comm-free row-partitioned SpMV.  x stays distributed: this rank's
+    slice lives in a libnest-owned buffer every peer maps (CUDA IPC), and the
+    SpMV's simd lanes gather x[c] from the owner's slice over NVLink -- no
+    all-gather.  torch.distributed only exchanges the IPC handle blobs.
+
+    ``local_slices``: single-process form (tests): a list of nranks CUDA tensors
+    (xchunk doubles each) standing for the ranks' slices; no IPC, no barrier."""
+
+    def __init__(self, ncols_global: int, group=None, *, nranks=None, rank=None, local_slices=None):
+        torch = _torch()
+        self._torch = torch
+        self._h = ctypes.c_void_p()
+        if local_slices is not None:
+            self.nranks, self.rank = int(nranks), int(rank)
+            xc = x_chunk(ncols_global, self.nranks)
+            if len(local_slices) != self.nranks:
+                raise ValueError("need one slice per rank")
+            arr = (ctypes.c_void_p * self.nranks)(*[_dev(t, torch.float64, xc, f"slice {r}").value if xc else None
+                                                    for r, t in enumerate(local_slices)])
+            self._keep = list(local_slices)
+            check(N.nest_xpeer_create_local(self.nranks, self.rank, ncols_global, arr, ctypes.byref(self._h)),
+                  "nest_xpeer_create_local")
+            return
+        import torch.distributed as dist
+        self.rank = dist.get_rank(group)
+        self.nranks = dist.get_world_size(group)
+        nb = int(N.nest_xpeer_handle_bytes())
+        blob = (ctypes.c_uint8 * nb)()
+        check(N.nest_xpeer_create(self.nranks, self.rank, ncols_global, ctypes.byref(self._h), blob),
+              "nest_xpeer_create")
+        blobs = [None] * self.nranks
+        dist.all_gather_object(blobs, bytes(blob), group=group)
+        allb = (ctypes.c_uint8 * (nb * self.nranks)).from_buffer_copy(b"".join(blobs))
+        check(N.nest_xpeer_open(self._h, allb), "nest_xpeer_open")
+
+    @property
+    def xchunk(self) -> int:
+        return int(N.nest_xpeer_xchunk(self._h))
+
+    def local_x(self):
+        """This rank's x slice (library-owned device memory) as a borrowed pointer."""
+        return N.nest_xpeer_local_x(self._h)
+
+    def set_local_x(self, x_local, stream=None):
+        """Copy this rank's part of x (a CUDA tensor, >= its slice length) into
+        its library-owned slice, stream-ordered (device to device)."""
+        torch = self._torch
+        check(N.nest_xpeer_set_x(self._h, _dev(x_local, torch.float64, None, "x_local"), x_local.numel(),
+                                 _stream(stream)), "nest_xpeer_set_x")
+
+    def barrier(self, stream=None):
+        check(N.nest_xpeer_barrier(self._h, _stream(stream)), "nest_xpeer_barrier")
+
+    def spmv_csr_f64(self, nrows_global, rowptr, colind, val, y_local=None, *, stream=None, **cfg):
+        """barrier; y_local = A[local rows] @ x gathering x from the owners' slices; barrier."""
+        torch = self._torch
+        nrows_local = rowptr.numel() - 1
+        nnz = val.numel()
+        if y_local is None:
+            y_local = torch.empty(nrows_local, dtype=torch.float64, device=val.device)
+        d = make_desc(**cfg)
+        check(N.nest_spmv_csr_f64_xpeer(ctypes.byref(d), self._h, nrows_global, nrows_local, nnz,
+                                        _dev(rowptr, torch.int64, nrows_local + 1, "rowptr"),
+                                        _dev(colind, torch.int32, nnz, "colind"),
+                                        _dev(val, torch.float64, nnz, "val"),
+                                        _dev(y_local, torch.float64, nrows_local, "y_local"),
+                                        _stream(stream)),
+              "nest_spmv_csr_f64_xpeer")
+        return y_local
+
+    def close(self):
+        if self._h:
+            check(N.nest_xpeer_destroy(self._h), "nest_xpeer_destroy")
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
