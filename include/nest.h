@@ -259,6 +259,36 @@ nest_status nest_spmv_csr_f64_dist(const nest_desc *desc, nest_comm *comm, int64
                                    const double *val, const double *x_local, double *x_full,
                                    double *y_local, void *stream);
 
+/* ---- NEXT-3: several parallel regions with their own simdlen in ONE kernel ----
+ * PAPER.md:511-513 ("the size could differ between parallel regions") and
+ * PAPER.md:686-698.  Every team runs regions[0..nregions) in order; region k
+ * partitions the team into SIMD groups of regions[k].simdlen lanes, re-divides
+ * the sharing space among its T / simdlen groups (global fallback when the
+ * region's payload does not fit) and ends with the team
+ * barrier of the end of a parallel region.  Teams are independent, so a region
+ * must not read what another team writes in an earlier region.  `desc` gives
+ * the team geometry (num_teams: 0 = one resident league; threads_per_team;
+ * sharing_bytes); its simdlen and mode are validated but unused; reduce must be
+ * SUM, outer_unroll 1, flags and team_chunk 0.  Each region's output is
+ * bit-identical to the stand-alone entry point at the same simdlen and mode. */
+#define NEST_MAX_REGIONS 4
+typedef enum {
+    NEST_REGION_SPMV_CSR_F64 = 0,       /* n = {nrows, ncols, nnz}; in = {rowptr, colind, val, x}; out = {y} */
+    NEST_REGION_BATCHED_MATVEC_F32 = 1, /* n = {batch, m, n}; in = {A, x}; out = {y} */
+    NEST_REGION_NESTED_STENCIL_F64 = 2  /* n = {nouter, L, 0}; in = {in, coef, w}; out = {out, visits or NULL} */
+} nest_region_kind;
+typedef struct {
+    int32_t kind;        /* nest_region_kind */
+    int32_t simdlen;     /* this region's SIMD group size: 1, 2, 4, 8, 16, 32 */
+    int32_t mode;        /* NEST_MODE_SPMD / GENERIC_SMEM / GENERIC_SHFL */
+    int32_t blocked;     /* 1: blocked team schedule (as NEST_F_BLOCKED), 0: cyclic */
+    int64_t n[3];        /* extents (per kind, above) */
+    const void *in[4];   /* device input arrays (per kind) */
+    void *out[2];        /* device output arrays (per kind) */
+} nest_region;
+nest_status nest_region_program(const nest_desc *desc, const nest_region *regions, int32_t nregions,
+                                void *stream);
+
 /* ---- NEXT-4: comm-free row-partitioned SpMV over peer memory ----
  * Same row and x partition as nest_spmv_csr_f64_dist, but x is never gathered:
  * every rank keeps its x slice (xchunk = ceil(ncols_global / nranks) doubles) in

@@ -39,6 +39,16 @@ class nest_desc(ctypes.Structure):
                 ("team_chunk", ctypes.c_int32), ("reserved", ctypes.c_int32)]
 
 
+NEST_MAX_REGIONS = 4
+NEST_REGION_SPMV_CSR_F64, NEST_REGION_BATCHED_MATVEC_F32, NEST_REGION_NESTED_STENCIL_F64 = 0, 1, 2
+
+
+class nest_region(ctypes.Structure):
+    _fields_ = [("kind", ctypes.c_int32), ("simdlen", ctypes.c_int32), ("mode", ctypes.c_int32),
+                ("blocked", ctypes.c_int32), ("n", ctypes.c_int64 * 3), ("in_", ctypes.c_void_p * 4),
+                ("out", ctypes.c_void_p * 2)]
+
+
 class nest_plan_info(ctypes.Structure):
     _fields_ = [("grid", ctypes.c_int32), ("block", ctypes.c_int32),
                 ("groups_per_team", ctypes.c_int32), ("slot_bytes", ctypes.c_int32),
@@ -69,6 +79,7 @@ SIGNATURES = {
     "nest_comm_init": (_st, [_vp, _i32, _i32, ctypes.POINTER(_vp)]),
     "nest_comm_destroy": (_st, [_vp]),
     "nest_spmv_csr_f64_dist": (_st, [_D, _vp, _i64, _i64, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _vp]),
+    "nest_region_program": (_st, [_D, ctypes.POINTER(nest_region), _i32, _vp]),
     "nest_xpeer_handle_bytes": (_sz, []),
     "nest_xpeer_create": (_st, [_i32, _i32, _i64, ctypes.POINTER(_vp), _vp]),
     "nest_xpeer_open": (_st, [_vp, _vp]),

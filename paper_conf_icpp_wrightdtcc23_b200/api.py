@@ -209,3 +209,51 @@ def l2_flush(buf, *, stream=None) -> None:
 
 def shutdown() -> None:
     check(N.nest_shutdown(), "nest_shutdown")
+
+
+def region_program(regions, *, stream=None, **team_cfg):
+    """NEXT-3: run up to NEST_MAX_REGIONS parallel regions, each with its own
+    simdlen and mode, inside ONE kernel.
+
+    ``regions``: dicts with ``kind`` in {"spmv", "batched", "stencil"},
+    ``simdlen``, ``mode`` (default "spmd"), ``blocked`` (default False) and the
+    kind's tensors -- spmv: rowptr, colind, val, x, y (ncols = x.numel());
+    batched: A, x, y, batch, m, n; stencil: inp, coef, w, out, nouter, L, visits
+    (optional).  ``team_cfg``: threads_per_team, num_teams, sharing_bytes."""
+    torch = _torch()
+    arr = (N.nest_region * len(regions))()
+    for k, r in enumerate(regions):
+        g = arr[k]
+        g.simdlen = r["simdlen"]
+        m = r.get("mode", "spmd")
+        g.mode = MODES[m] if isinstance(m, str) else int(m)
+        g.blocked = int(bool(r.get("blocked", False)))
+        kind = r["kind"]
+        if kind == "spmv":
+            nrows, nnz = r["rowptr"].numel() - 1, r["val"].numel()
+            ncols = r["x"].numel()
+            g.kind = N.NEST_REGION_SPMV_CSR_F64
+            g.n[:] = [nrows, ncols, nnz]
+            g.in_[:] = [_dev(r["rowptr"], torch.int64, nrows + 1, "rowptr"), _dev(r["colind"], torch.int32, nnz, "colind"),
+                        _dev(r["val"], torch.float64, nnz, "val"), _dev(r["x"], torch.float64, ncols, "x")]
+            g.out[0] = _dev(r["y"], torch.float64, nrows, "y")
+        elif kind == "batched":
+            b, mm, n = r["batch"], r["m"], r["n"]
+            g.kind = N.NEST_REGION_BATCHED_MATVEC_F32
+            g.n[:] = [b, mm, n]
+            g.in_[0] = _dev(r["A"], torch.float32, b * mm * n, "A")
+            g.in_[1] = _dev(r["x"], torch.float32, b * n, "x")
+            g.out[0] = _dev(r["y"], torch.float32, b * mm, "y")
+        elif kind == "stencil":
+            no, L = r["nouter"], r["L"]
+            g.kind = N.NEST_REGION_NESTED_STENCIL_F64
+            g.n[:] = [no, L, 0]
+            g.in_[:] = [_dev(r["inp"], torch.float64, no * L + 2, "in"), _dev(r["coef"], torch.float64, L, "coef"),
+                        _dev(r["w"], torch.float64, no, "w"), None]
+            g.out[0] = _dev(r["out"], torch.float64, no, "out")
+            v = r.get("visits")
+            g.out[1] = _dev(v, torch.int64, 1, "visits") if v is not None else None
+        else:
+            raise ValueError(f"unknown region kind {kind!r}")
+    d = make_desc(**team_cfg)
+    check(N.nest_region_program(ctypes.byref(d), arr, len(regions), _stream(stream)), "nest_region_program")

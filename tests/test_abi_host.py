@@ -121,3 +121,18 @@ def test_team_chunk_validation():
     assert e.value.status == N.NEST_ERR_INVALID_ARG
     info = P.plan(1000, 24, team_chunk=100, blocked=True, num_teams=4)
     assert info["grid"] == 4
+
+
+def test_region_program_validates_before_any_device_call():
+    d = P.make_desc()
+    regs = (N.nest_region * 5)()
+    assert N.nest_region_program(ctypes.byref(d), regs, 0, None) == N.NEST_ERR_INVALID_ARG
+    assert N.nest_region_program(ctypes.byref(d), regs, 5, None) == N.NEST_ERR_INVALID_ARG
+    regs[0].kind, regs[0].simdlen = N.NEST_REGION_SPMV_CSR_F64, 3      # not a divisor of the warp
+    assert N.nest_region_program(ctypes.byref(d), regs, 1, None) == N.NEST_ERR_INVALID_ARG
+    regs[0].simdlen, regs[0].kind = 8, 7                                # unknown body
+    assert N.nest_region_program(ctypes.byref(d), regs, 1, None) == N.NEST_ERR_INVALID_ARG
+    regs[0].kind, regs[0].n[0] = N.NEST_REGION_SPMV_CSR_F64, 10         # rows but NULL arrays
+    assert N.nest_region_program(ctypes.byref(d), regs, 1, None) == N.NEST_ERR_INVALID_ARG
+    d.reduce = N.NEST_REDUCE_MAX
+    assert N.nest_region_program(ctypes.byref(d), regs, 1, None) == N.NEST_ERR_UNSUPPORTED

@@ -1,0 +1,87 @@
+"""NEXT-3: parallel regions with different simdlen in one kernel
+(PAPER.md:511-513, 686-698).  Each region's output is bit-identical to the
+stand-alone entry point at the same simdlen and mode, the stencil's visit
+counter equals nouter, and a tiny sharing space forces some regions onto the
+global fallback without changing any result."""
+import numpy as np
+import pytest
+
+import oracle
+from nestgen import recipes as R
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def P():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_icpp_wrightdtcc23_b200 as P
+    return P
+
+
+def bits(t):
+    a = t.cpu().numpy()
+    return a.view(np.int64 if a.dtype == np.float64 else np.int32)
+
+
+@pytest.fixture(scope="module")
+def data():
+    spec = R.SpmvSpec("prog", 4343, 20_000, 20_000, 0, 40, band_w=900, far_den=8)
+    rp, col, val, x = R.spmv_inputs(spec)
+    ys, ya = oracle.spmv_csr_f64(rp, col, val, x)
+    B = 777
+    A, xb = R.batched_inputs(B)
+    N, L = 5003, 16
+    inp, coef, w = R.stencil_inputs(N, L)
+    cu = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
+    return dict(spmv=[cu(a) for a in (rp, col, val, x)], ys=ys, ya=ya, B=B, A=cu(A), xb=cu(xb),
+                N=N, L=L, st=[cu(a) for a in (inp, coef, w)])
+
+
+COMBOS = [  # (spmv S, mode), (batched S, mode), (stencil S, mode)
+    ((8, "generic_smem"), (4, "spmd"), (32, "generic_shfl")),
+    ((1, "spmd"), (32, "generic_smem"), (2, "generic_smem")),
+    ((32, "spmd"), (2, "generic_shfl"), (16, "spmd")),
+    ((4, "generic_shfl"), (16, "generic_smem"), (1, "spmd")),
+]
+
+
+@pytest.mark.parametrize("combo", COMBOS)
+@pytest.mark.parametrize("T,sharing,teams", [(256, 0, 0), (128, 64, 0), (1024, 2048, 7)])
+def test_region_program_matches_standalone(P, data, combo, T, sharing, teams):
+    (s1, m1), (s2, m2), (s3, m3) = combo
+    y = torch.empty(data["spmv"][0].numel() - 1, dtype=torch.float64, device="cuda")
+    yb = torch.empty(data["B"] * 64, dtype=torch.float32, device="cuda")
+    out = torch.empty(data["N"], dtype=torch.float64, device="cuda")
+    visits = torch.zeros(1, dtype=torch.int64, device="cuda")
+    rp, col, val, x = data["spmv"]
+    inp, coef, w = data["st"]
+    regions = [
+        dict(kind="spmv", simdlen=s1, mode=m1, blocked=True, rowptr=rp, colind=col, val=val, x=x, y=y),
+        dict(kind="batched", simdlen=s2, mode=m2, A=data["A"], x=data["xb"], y=yb, batch=data["B"], m=64, n=64),
+        dict(kind="stencil", simdlen=s3, mode=m3, blocked=bool(teams), inp=inp, coef=coef, w=w, out=out,
+             nouter=data["N"], L=data["L"], visits=visits),
+    ]
+    P.region_program(regions, threads_per_team=T, sharing_bytes=sharing, num_teams=teams)
+    ref_y = P.spmv_csr_f64(rp, col, val, x, simdlen=s1, mode=m1)
+    ref_yb = P.batched_matvec_f32(data["A"], data["xb"], data["B"], simdlen=s2, mode=m2)
+    ref_out = P.nested_stencil_f64(inp, coef, w, data["N"], data["L"], simdlen=s3, mode=m3)
+    assert np.array_equal(bits(y), bits(ref_y))
+    assert np.array_equal(bits(yb), bits(ref_yb))
+    assert np.array_equal(bits(out), bits(ref_out))
+    assert int(visits.item()) == data["N"]
+    assert np.all(np.abs(y.cpu().numpy() - data["ys"]) <= 1e-12 * data["ya"])
+
+
+def test_region_program_rejects(P, data):
+    rp, col, val, x = data["spmv"]
+    y = torch.empty(rp.numel() - 1, dtype=torch.float64, device="cuda")
+    r = dict(kind="spmv", simdlen=8, rowptr=rp, colind=col, val=val, x=x, y=y)
+    with pytest.raises(P.NestError):
+        P.region_program([r] * 5)                         # more than NEST_MAX_REGIONS
+    with pytest.raises(P.NestError):
+        P.region_program([dict(r, simdlen=3)])            # not a divisor of the warp
+    with pytest.raises(P.NestError):
+        P.region_program([r], reduce="max")               # SUM only
