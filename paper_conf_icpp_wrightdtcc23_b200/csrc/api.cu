@@ -113,8 +113,10 @@ static nest_status plan_core(const nest_desc* d, int64_t outer, int32_t K, int32
         return fail(NEST_ERR_INVALID_ARG, "NEST_F_VEC_QUAD applies to the CSR SpMV only");
     if ((d->flags & NEST_F_VEC_QUAD) && !(d->flags & NEST_F_VEC128))
         return fail(NEST_ERR_INVALID_ARG, "NEST_F_VEC_QUAD needs NEST_F_VEC128");
-    if ((d->flags & NEST_F_VEC128) && (d->x_halo > 0 || (d->flags & NEST_F_STAGED)))
-        return fail(NEST_ERR_UNSUPPORTED, "NEST_F_VEC128 combines with the cyclic or blocked schedule only");
+    if ((d->flags & NEST_F_VEC128) && (d->flags & NEST_F_STAGED))
+        return fail(NEST_ERR_UNSUPPORTED, "NEST_F_VEC128 does not combine with NEST_F_STAGED");
+    if ((d->flags & NEST_F_VEC_QUAD) && d->x_halo > 0)
+        return fail(NEST_ERR_UNSUPPORTED, "x_halo takes scalar or pair loads (not NEST_F_VEC_QUAD)");
     if ((d->flags & NEST_F_STAGED) && T < 128)
         return fail(NEST_ERR_INVALID_ARG,
                     "NEST_F_STAGED needs threads_per_team >= 128 (producer, 2 gather and >= 1 consumer warps)");
@@ -142,25 +144,43 @@ static nest_status plan_core(const nest_desc* d, int64_t outer, int32_t K, int32
         q.x_halo = d->x_halo;   // stage sizes and grid: plan_spmv_staged (needs nnz)
         q.grid = d->num_teams;
     } else if (d->x_halo > 0) {
-        // x window (spmv_xwin.cuh): ring of XW = 2R + 2H doubles (even), R = G*U rows per
-        // chunk, plus a double-buffered rowptr stage; always a persistent block schedule.
-        const int64_t R = (int64_t)q.groups * U;
-        const int64_t xw = (2 * R + 2 * (int64_t)d->x_halo + 1) & ~(int64_t)1;
-        const int64_t bytes = xw * 8 + 2 * (R + 1) * 8 + q.smem_bytes;
-        if (bytes > kMaxDynSmem)
+        // x window (spmv_xwin.cuh): ring of XW = 2R + 2H doubles, R = G*U*KB rows per
+        // chunk (even), H = x_halo rounded up to even; KB: the most rows per chunk
+        // whose ring still lets 2048 / T teams share an SM, else the fewest that fit.
+        const int64_t H = ((int64_t)d->x_halo + 1) & ~(int64_t)1;
+        const int64_t per_sm = kMaxThreadsPerSm / T > 0 ? kMaxThreadsPerSm / T : 1;
+        const int64_t budget = kSmemPerSm / per_sm - kSmemReservedPerBlock;
+        int64_t kb = 0, bytes = 0;
+        for (int64_t k = 16; k >= 1; k >>= 1) {
+            const int64_t R = (int64_t)q.groups * U * k;
+            const int64_t b = (2 * R + 2 * H) * 8 + 16 + q.smem_bytes;
+            if (R % 2 == 0 && b <= budget && b <= kMaxDynSmem) {
+                kb = k, bytes = b;
+                break;
+            }
+        }
+        for (int64_t k = 1; kb == 0 && k <= 16; k <<= 1) {
+            const int64_t R = (int64_t)q.groups * U * k;
+            const int64_t b = (2 * R + 2 * H) * 8 + 16 + q.smem_bytes;
+            if (R % 2 == 0 && b <= kMaxDynSmem) kb = k, bytes = b;
+        }
+        if (kb == 0)
             return fail(NEST_ERR_UNSUPPORTED,
-                        "x_halo %d with %lld rows per chunk needs %lld B of shared memory (max %d)",
-                        d->x_halo, (long long)R, (long long)bytes, kMaxDynSmem);
-        q.x_halo = d->x_halo;
-        q.xw = (int32_t)xw;
+                        "x_halo %d with %lld rows per batch needs more than %d B of shared memory",
+                        d->x_halo, (long long)q.groups * U, kMaxDynSmem);
+        const int64_t R = (int64_t)q.groups * U * kb;
+        q.x_halo = (int32_t)H;
+        q.kb = (int32_t)kb;
+        q.xw = (int32_t)(2 * R + 2 * H);
         q.smem_bytes = (int32_t)bytes;
+        const int64_t chunks = (outer + R - 1) / R;
         if (d->num_teams > 0) {
             q.grid = d->num_teams;
         } else {
             int64_t resident = 0;
             nest_status s = resident_blocks(T, q.smem_bytes, &resident);
             if (s != NEST_OK) return s;
-            q.grid = (int32_t)(needed < resident ? needed : resident);
+            q.grid = (int32_t)(chunks < resident ? (chunks > 0 ? chunks : 1) : resident);
         }
     } else if (d->num_teams > 0) {
         q.grid = d->num_teams;
@@ -337,7 +357,12 @@ NEST_API nest_status nest_spmv_csr_f64(const nest_desc* desc, int64_t nrows, int
         return fail(NEST_ERR_UNSUPPORTED, "NEST_F_VEC128 needs 16-byte aligned val and %d-byte aligned colind",
                     (p.flags & NEST_F_VEC_QUAD) ? 16 : 8);
     if (staged) return launch_spmv_staged(p, nrows, ncols, nnz, rowptr, colind, val, x, y, fb, as_stream(stream));
-    if (p.x_halo > 0) return launch_spmv_xwin(p, nrows, ncols, rowptr, colind, val, x, y, fb, as_stream(stream));
+    if (p.x_halo > 0) {
+        if (reinterpret_cast<uintptr_t>(x) & 15) return fail(NEST_ERR_UNSUPPORTED, "x_halo needs 16-byte aligned x");
+        if ((p.flags & NEST_F_VEC128) && (nnz >= ((int64_t)1 << 31) - 8 || nrows >= ((int64_t)1 << 31) - 8))
+            return fail(NEST_ERR_UNSUPPORTED, "x_halo with NEST_F_VEC128 needs nnz, nrows < 2^31");
+        return launch_spmv_xwin(p, nrows, ncols, nnz, rowptr, colind, val, x, y, fb, as_stream(stream));
+    }
     return launch_spmv(p, (p.flags & NEST_F_STREAM_HINTS) != 0, nrows, rowptr, colind, val, x, y, fb,
                        as_stream(stream), nnz);
 }
@@ -380,6 +405,8 @@ NEST_API nest_status nest_spmv_csr_f64_hostio(const nest_desc* desc, int64_t nro
     const bool staged = (p.flags & NEST_F_STAGED) != 0;
     if (staged && (s = plan_spmv_staged(&p, nrows, nnz, desc->sharing_bytes ? desc->sharing_bytes : kDefaultSharing)) != NEST_OK)
         return s;
+    if (p.x_halo > 0 && (p.flags & NEST_F_VEC128) && (nnz >= ((int64_t)1 << 31) - 8 || nrows >= ((int64_t)1 << 31) - 8))
+        return fail(NEST_ERR_UNSUPPORTED, "x_halo with NEST_F_VEC128 needs nnz, nrows < 2^31");
     unsigned char* fb = nullptr;
     if ((s = prepare_fallback(p, &fb)) != NEST_OK) return s;
     cudaStream_t st = as_stream(stream);
@@ -390,7 +417,7 @@ NEST_API nest_status nest_spmv_csr_f64_hostio(const nest_desc* desc, int64_t nro
         (ncols && (e = cudaMemcpyAsync(d_x, h_x, (size_t)ncols * 8, cudaMemcpyHostToDevice, st))))
         return cuda_fail(e, "host->device copy");
     s = staged ? launch_spmv_staged(p, nrows, ncols, nnz, d_rowptr, d_col, d_val, d_x, d_y, fb, st)
-        : p.x_halo > 0 ? launch_spmv_xwin(p, nrows, ncols, d_rowptr, d_col, d_val, d_x, d_y, fb, st)
+        : p.x_halo > 0 ? launch_spmv_xwin(p, nrows, ncols, nnz, d_rowptr, d_col, d_val, d_x, d_y, fb, st)
                      : launch_spmv(p, (p.flags & NEST_F_STREAM_HINTS) != 0, nrows, d_rowptr, d_col, d_val,
                                    d_x, d_y, fb, st, nnz);
     if (s != NEST_OK) return s;

@@ -29,7 +29,7 @@ struct Plan {
     int64_t outer = 0;
     int64_t chunk = 0;     // NEST_F_BLOCKED: outer iterations per team chunk (a multiple of G)
     int32_t x_halo = 0;    // SpMV x window half-width (0 = none)
-    int32_t xw_log2 = 0;   // ring of 2^xw_log2 doubles
+    int32_t kb = 1;        // x window: batches of U rows per group per chunk
     // NEST_F_STAGED pipeline (spmv_staged.cuh)
     int32_t xw = 0;        // x ring capacity in doubles (even; 0 = no window)
     int32_t nb = 0;        // stage capacity in nonzeros
@@ -69,7 +69,7 @@ int32_t laplace_payload(int32_t U);
 nest_status launch_spmv(const Plan& p, bool hints, int64_t nrows, const int64_t* rowptr,
                         const int32_t* col, const double* val, const double* x, double* y,
                         unsigned char* fb, cudaStream_t st, int64_t nnz);
-nest_status launch_spmv_xwin(const Plan& p, int64_t nrows, int64_t ncols, const int64_t* rowptr,
+nest_status launch_spmv_xwin(const Plan& p, int64_t nrows, int64_t ncols, int64_t nnz, const int64_t* rowptr,
                              const int32_t* col, const double* val, const double* x, double* y,
                              unsigned char* fb, cudaStream_t st);
 // NEST_F_STAGED: finish the plan from the matrix shape (stage sizes, grid) and launch.

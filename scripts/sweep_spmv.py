@@ -55,7 +55,7 @@ def main():
                                               for bl in map(int, a.blocked.split(","))
                                               for vc in map(int, a.vec.split(","))
                                               for ck in map(int, a.chunks.split(","))]:
-                        if vc and xh:
+                        if vc == 2 and xh:
                             continue
                         cfg = dict(simdlen=S, mode=mode, outer_unroll=U, stream_hints=bool(h), threads_per_team=T,
                                    x_halo=xh, staged=bool(sg), blocked=bool(bl), vec128=vc >= 1, quad=vc == 2, team_chunk=ck if bl else 0)
