@@ -233,7 +233,10 @@ nest_status nest_probe_mapping(const nest_desc *desc, int32_t *out_map, int64_t 
 nest_status nest_csr_validate(int64_t nrows, int64_t ncols, int64_t nnz, const int64_t *rowptr,
                               const int32_t *colind, int32_t *d_bad, void *stream);
 
-/* Bench utility: overwrite `bytes` of device memory at `buf` (flushes L2). */
+/* Bench utility: flush L2.  Overwrites `bytes` of device memory at `buf`, then
+ * reads back its first half, so that L2 ends up holding only clean lines
+ * unrelated to any later kernel (no dirty write-backs inside the next, timed,
+ * kernel).  `bytes` should exceed twice the L2 size (bench: 512 MiB). */
 nest_status nest_util_l2_flush(void *buf, size_t bytes, void *stream);
 
 /* ---- a12: row-partitioned multi-GPU SpMV (north_star; the paper is single-GPU) ----

@@ -1,5 +1,6 @@
 // api.cu -- the C ABI of include/nest.h: validation, the a1 planner, the
 // library-owned sharing-space fallback and the single-GPU entry points.
+#include <cstdlib>
 #include <cuda_runtime.h>
 
 #include <climits>
@@ -280,6 +281,17 @@ __global__ void l2_flush_kernel(uint4* __restrict__ buf, size_t n16, uint32_t sa
         buf[i] = make_uint4(salt, (uint32_t)i, salt ^ 0x9e3779b9u, (uint32_t)(i >> 32));
 }
 
+// Second flush phase: read the first half of the buffer (written earliest, so
+// no longer resident) -- L2 ends up holding only clean lines, and the dirty
+// lines of the write phase are written back here rather than inside the next
+// (timed) kernel.
+__global__ void l2_clean_kernel(const uint4* __restrict__ buf, size_t n16, uint32_t* sink) {
+    const size_t stride = (size_t)gridDim.x * blockDim.x;
+    uint32_t acc = 0;
+    for (size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < n16; i += stride) acc ^= __ldcg(buf + i).y;
+    if (acc == 0x9e3779b9u && sink) *sink = acc;
+}
+
 }  // namespace nest
 
 using namespace nest;
@@ -505,6 +517,9 @@ NEST_API nest_status nest_util_l2_flush(void* buf, size_t bytes, void* stream) {
     const size_t n16 = bytes / 16;
     if (n16 == 0) return NEST_OK;
     l2_flush_kernel<<<1184, 512, 0, as_stream(stream)>>>(static_cast<uint4*>(buf), n16, salt++);
+    const char* ce = std::getenv("NEST_FLUSH_CLEAN");   // 0: write phase only (A/B experiments)
+    if (!ce || std::atoi(ce) != 0)
+        l2_clean_kernel<<<1184, 512, 0, as_stream(stream)>>>(static_cast<const uint4*>(buf), n16 / 2, nullptr);
     const cudaError_t e = cudaGetLastError();
     return e == cudaSuccess ? NEST_OK : cuda_fail(e, "l2_flush launch");
 }

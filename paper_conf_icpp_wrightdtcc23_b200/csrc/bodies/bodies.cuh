@@ -23,6 +23,10 @@
 #ifndef NEST_VEC_UNROLL
 #define NEST_VEC_UNROLL 1
 #endif
+// tuples per lane issued as one predicated block by the 128-bit SpMV body
+#ifndef NEST_VEC_HEAD
+#define NEST_VEC_HEAD 2
+#endif
 
 namespace nest {
 
@@ -134,6 +138,7 @@ struct XPeer {
 template <bool HINTS, bool PIPE = false, class I = int64_t, class XA = XLocal>
 struct SpmvBody {
     using Acc = double;
+    using OuterIndex = I;   // launcher: I = int32_t only when spmv_index32()
     // I: index type of rows and nonzeros (int32_t when they fit: fewer registers)
     struct Loop {
         I trip;   // nonzeros in the row (TripCount)
@@ -218,6 +223,7 @@ struct SpmvVecBody {
     // I: index type of rows and nonzeros (int32_t when nnz and nrows < 2^31:
     // fewer registers, so two teams of 1024 fit an SM)
     using Acc = double;
+    using OuterIndex = I;   // launcher: I = int32_t only when spmv_index32()
     static constexpr int kLoopUnroll = NEST_VEC_UNROLL;   // V nonzeros per iteration already
     struct Loop {
         I base;         // rowptr[i]
@@ -249,15 +255,9 @@ struct SpmvVecBody {
         constexpr int kLog = V == 2 ? 1 : 2;
         return Loop{b, e > b ? (int32_t)(((e + V - 1) >> kLog) - (b >> kLog)) : 0, (int32_t)(e - b)};
     }
-    template <int OP>
-    __device__ __forceinline__ double accum(const Loop& L, int32_t j, double acc) const {
-        const I b = L.base;
-        const I e = b + L.len;
-        constexpr int kLog = V == 2 ? 1 : 2;
-        const I k0 = ((b >> kLog) + j) << kLog;   // first entry of the tuple
-        int32_t c[V];
-        double v[V];
-        if ((int64_t)k0 + V <= nnz) {
+    // the tuple starting at entry k0: 128-bit loads, scalar at the end of the arrays
+    __device__ __forceinline__ void load_tuple(I k0, int32_t (&c)[V], double (&v)[V]) const {
+        if (k0 + V <= (I)nnz) {
             if constexpr (V == 2) {
                 const int2 cc = HINTS ? ld_na(reinterpret_cast<const int2*>(col + k0))
                                       : __ldg(reinterpret_cast<const int2*>(col + k0));
@@ -279,15 +279,70 @@ struct SpmvVecBody {
         } else {
 #pragma unroll
             for (int q = 0; q < V; ++q) {
-                const I kq = (int64_t)k0 + q < nnz ? k0 + q : k0;
+                const I kq = k0 + q < (I)nnz ? k0 + q : k0;
                 c[q] = __ldg(col + kq);
                 v[q] = __ldg(val + kq);
             }
         }
+    }
+    template <int OP>
+    __device__ __forceinline__ double accum(const Loop& L, int32_t j, double acc) const {
+        const I b = L.base;
+        const I e = b + L.len;
+        constexpr int kLog = V == 2 ? 1 : 2;
+        const I k0 = ((b >> kLog) + j) << kLog;   // first entry of the tuple
+        int32_t c[V];
+        double v[V];
+        load_tuple(k0, c, v);
 #pragma unroll
         for (int q = 0; q < V; ++q)
             if (k0 + q >= b && k0 + q < e)
                 acc = Red<OP, double>::accum(acc, v[q], x(c[q]));
+        return acc;
+    }
+    // the lane's first kHeadIters tuples (j = id, id + S, ...) as one predicated
+    // block: all tuple loads, then all x gathers, then the folds in order
+    // (engine.cuh head_iters; measured 0.313 -> 0.293 ms on cfg2 at S = 2).
+    static constexpr int kHeadIters = V == 2 ? NEST_VEC_HEAD : 1;   // quads: 2 would spill (32 registers)
+    template <int OP, int S>
+    __device__ __forceinline__ double accum_head(const Loop& L, int32_t id, double acc) const {
+        constexpr int H = kHeadIters > 0 ? kHeadIters : 1;
+        const I b = L.base;
+        const I e = b + L.len;
+        constexpr int kLog = V == 2 ? 1 : 2;
+        int32_t c[H][V];
+        double v[H][V];
+#pragma unroll
+        for (int h = 0; h < H; ++h) {
+            const int32_t j = id + h * S;
+            const I k0 = ((b >> kLog) + j) << kLog;
+            if (j < L.trip && k0 + V <= (I)nnz) {   // one branch: the 128-bit tuple
+                load_tuple(k0, c[h], v[h]);
+            } else {                                         // predicated scalar loads (array end / idle)
+#pragma unroll
+                for (int q = 0; q < V; ++q) {
+                    const I kq = k0 + q < (I)nnz ? k0 + q : (I)nnz - 1;
+                    c[h][q] = j < L.trip ? __ldg(col + kq) : 0;
+                    v[h][q] = j < L.trip ? __ldg(val + kq) : 0.0;
+                }
+            }
+        }
+        double xv[H][V];
+#pragma unroll
+        for (int h = 0; h < H; ++h) {
+            const int32_t j = id + h * S;
+            const I k0 = ((b >> kLog) + j) << kLog;
+#pragma unroll
+            for (int q = 0; q < V; ++q) xv[h][q] = (j < L.trip && k0 + q >= b && k0 + q < e) ? x(c[h][q]) : 0.0;
+        }
+#pragma unroll
+        for (int h = 0; h < H; ++h) {
+            const int32_t j = id + h * S;
+            const I k0 = ((b >> kLog) + j) << kLog;
+#pragma unroll
+            for (int q = 0; q < V; ++q)
+                if (j < L.trip && k0 + q >= b && k0 + q < e) acc = Red<OP, double>::accum(acc, v[h][q], xv[h][q]);
+        }
         return acc;
     }
     __device__ __forceinline__ void epilogue(const Step& st, double total) const { y[st.i] = total; }

@@ -38,6 +38,14 @@ struct Plan {
     int32_t pipe_off = -1; // nest_kernel loop-bound pipeline ring offset in dynamic smem (-1 = off)
 };
 
+// 32-bit row / nonzero indices (and 32-bit outer-loop cursors, engine.cuh
+// outer_index) when every index and every schedule position fits with room to
+// spare: fewer instructions and registers per row.
+inline bool spmv_index32(const Plan& p, int64_t nnz) {
+    const int64_t lim = (int64_t)1 << 30;
+    return nnz < ((int64_t)1 << 31) - 8 && p.outer < lim && (int64_t)p.grid * p.chunk < lim;
+}
+
 // Record a thread-local error message and return `s`.
 nest_status fail(nest_status s, const char* fmt, ...) __attribute__((format(printf, 2, 3)));
 nest_status cuda_fail(cudaError_t e, const char* what);

@@ -50,7 +50,7 @@ static nest_status launch_spmv_t(const Plan& p, const int64_t* rowptr, const int
                                  const double* x, double* y, unsigned char* fb, cudaStream_t st, int64_t nnz,
                                  int64_t ahead, int64_t len) {
     // 32-bit row / nonzero indices when they fit (fewer registers)
-    if (nnz < ((int64_t)1 << 31) - 8 && p.outer < ((int64_t)1 << 31) - 8) {
+    if (spmv_index32(p, nnz)) {
         SpmvBody<HINTS, PIPE, int32_t> b{rowptr, col, val, x, y};
         b.nnz = nnz, b.pf_ahead = ahead, b.pf_len = len;
         return spmv_dispatch(p, b, fb, st);
@@ -66,7 +66,7 @@ nest_status launch_spmv_body(const Plan& p, bool hints, const int64_t* rowptr, c
     const bool pipe = p.pipe_off >= 0;
     if (p.flags & NEST_F_VEC128) {
         // 32-bit row / nonzero indices when they fit (fewer registers)
-        const bool i32 = nnz < ((int64_t)1 << 31) - 8 && p.outer < ((int64_t)1 << 31) - 8;
+        const bool i32 = spmv_index32(p, nnz);
         if (p.flags & NEST_F_VEC_QUAD) {
             if (i32) return spmv_dispatch(p, SpmvVecBody<false, 4, int32_t>{rowptr, col, val, x, y, nnz}, fb, st);
             return spmv_dispatch(p, SpmvVecBody<false, 4, int64_t>{rowptr, col, val, x, y, nnz}, fb, st);

@@ -228,8 +228,8 @@ NEST_API nest_status nest_spmv_csr_f64_xpeer(const nest_desc* desc, nest_xpeer* 
     if (nrows_local > 0 && (!rowptr || !y)) return fail(NEST_ERR_INVALID_ARG, "rowptr/y is NULL");
     if (nnz > 0 && (!colind || !val)) return fail(NEST_ERR_INVALID_ARG, "colind/val is NULL");
     const bool vec = (p.flags & NEST_F_VEC128) != 0;
-    const bool i32 = nnz < ((int64_t)1 << 31) - 8 && nrows_local < ((int64_t)1 << 31) - 8;
-    if (vec && !i32) return fail(NEST_ERR_UNSUPPORTED, "NEST_F_VEC128 (xpeer) needs nnz_local < 2^31");
+    const bool i32 = spmv_index32(p, nnz);
+    if (vec && !i32) return fail(NEST_ERR_UNSUPPORTED, "NEST_F_VEC128 (xpeer) needs nnz_local < 2^31, nrows_local < 2^30");
     if (vec && ((reinterpret_cast<uintptr_t>(val) & 15) || (reinterpret_cast<uintptr_t>(colind) & 7)))
         return fail(NEST_ERR_UNSUPPORTED, "NEST_F_VEC128 needs 16-byte aligned val and 8-byte aligned colind");
     unsigned char* fb = nullptr;

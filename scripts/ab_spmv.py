@@ -1,0 +1,44 @@
+"""A/B timing of SpMV configurations on cfg2 (developer experiment, not the bench):
+alternates L2-flush modes (NEST_FLUSH_CLEAN) and configurations in one process.
+python scripts/ab_spmv.py [rounds]"""
+import os
+import statistics
+import sys
+
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import paper_conf_icpp_wrightdtcc23_b200 as P  # noqa: E402
+from nestgen import recipes as R  # noqa: E402
+
+spec = R.CFG2
+rp, col, val = R.spmv_matrix(spec)
+x = R.spmv_x(spec)
+t = [torch.from_numpy(v).cuda() for v in (rp, col, val, x)]
+y = torch.empty(spec.nrows, dtype=torch.float64, device="cuda")
+flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
+CFGS = {
+    "S2 bv": dict(simdlen=2, threads_per_team=1024, blocked=True, vec128=True),
+    "S1 bv": dict(simdlen=1, threads_per_team=1024, blocked=True, vec128=True),
+    "S2 b": dict(simdlen=2, threads_per_team=1024, blocked=True),
+    "S1 cyc256": dict(simdlen=1, threads_per_team=256),
+}
+rounds = int(sys.argv[1]) if len(sys.argv) > 1 else 3
+res = {}
+for r in range(rounds):
+    for clean in ("0", "1"):
+        os.environ["NEST_FLUSH_CLEAN"] = clean
+        for name, cfg in CFGS.items():
+            ts = []
+            for _ in range(12):
+                P.l2_flush(flush)
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record()
+                P.spmv_csr_f64(*t, y, **cfg)
+                e1.record()
+                ts.append((e0, e1))
+            torch.cuda.synchronize()
+            ms = [a.elapsed_time(b) for a, b in ts][2:]
+            res.setdefault((name, clean), []).append(statistics.median(ms))
+for (name, clean), v in sorted(res.items()):
+    print(f"{name:12s} clean={clean}  medians {' '.join(f'{m:.4f}' for m in v)}")
