@@ -10,3 +10,4 @@ for v in "2 best" "1 s1"; do
   ncu -i /tmp/$2.ncu-rep --page raw --csv > gpurun_out/prof/$2_raw.csv 2>/dev/null
   python scripts/ncu_summary.py /tmp/$2.ncu-rep > gpurun_out/prof/$2_summary.txt 2>&1
 done
+python scripts/launch_summary.py gpurun_out/prof/launches.csv > gpurun_out/prof/launches_summary.txt 2>&1
