@@ -417,6 +417,13 @@ def run_gpu(args, rank, world, local_rank):
                 "gpu_launches_detail": ("per step: barrier + SpMV + barrier kernels (+ l2_flush outside the events)"
                                         if head == "xpeer" else "per step: SpMV kernel + NCCL all-gather"),
                 "clocks": clocks, "e2e": e2e}
+        peak, peak_src = peaks()
+        per_gpu = line["value"] / world
+        line["roofline"] = {"bound": "hbm", "achieved": per_gpu, "peak": peak, "unit": "GB/s",
+                            "frac": per_gpu / peak, "traffic": None, "peak_source": peak_src,
+                            "kernel": f"nest_kernel<S={cfg['simdlen']},{cfg['mode']},SUM,U=1,SpmvVecBody<0,2,int,"
+                                      f"{'XPeer' if head == 'xpeer' else 'XLocal'}>>",
+                            "note": "per GPU: algorithmic bytes of all ranks / world / max-over-ranks step time"}
         print(json.dumps(line), flush=True)
     if "xpeer" in res:
         xp.close()

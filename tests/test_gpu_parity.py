@@ -212,8 +212,39 @@ def test_spmv_cfg2_full_size_sampled(P):
                 y = host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, outer_unroll=U, stream_hints=hints))
                 for s, (yr, ar) in ref.items():
                     assert_close(y[s:s + 64], yr, ar, 1e-12)
+    # the bench's candidate set (bench.CANDIDATES: blocked teams of 1024, 128-bit pairs / quads, the
+    # lean SPMD driver) including the headline and the simdlen-1 comparison point, plus team chunks
+    for S, mode, flags, chunk in ((2, "spmd", "bv", 0), (1, "spmd", "bv", 0), (1, "spmd", "bq", 0),
+                                  (2, "spmd", "bq", 0), (4, "spmd", "bv", 0), (2, "spmd", "b", 0),
+                                  (1, "spmd", "b", 0), (2, "generic_smem", "b", 0), (2, "spmd", "bv", 2048),
+                                  (8, "generic_shfl", "bv", 4096)):
+        y = host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, threads_per_team=1024, blocked="b" in flags,
+                                vec128="v" in flags or "q" in flags, quad="q" in flags, team_chunk=chunk))
+        for s, (yr, ar) in ref.items():
+            assert_close(y[s:s + 64], yr, ar, 1e-12)
     del t
     torch.cuda.empty_cache()
+
+
+def test_spmv_g100_and_uniform_full_size_sampled(P):
+    """The 100M-nnz gate matrix (G100) and the all-far cfg2 variant at full size in
+    the bench headline configuration: sampled 64-row windows against the oracle
+    on the same rows regenerated independently (R3 tolerance)."""
+    for spec in (R.G100, R.CFG2_UNIFORM):
+        rp, col, val = R.spmv_matrix(spec)
+        x = R.spmv_x(spec)
+        t = [dev(rp), dev(col), dev(val), dev(x)]
+        del rp, col, val
+        rng = np.random.default_rng(11)
+        starts = np.concatenate([[0, spec.nrows - 64], rng.integers(0, spec.nrows - 64, 16)])
+        for S, flags in ((2, "bv"), (1, "bv")):
+            y = host(P.spmv_csr_f64(*t, simdlen=S, threads_per_team=1024, blocked=True, vec128=True))
+            for s in starts:
+                rpl, cl, vl = R.spmv_matrix(spec, row_begin=int(s), nrows=64)
+                yr, ar = oracle.spmv_csr_f64(rpl, cl, vl, x)
+                assert_close(y[s:s + 64], yr, ar, 1e-12)
+        del t
+        torch.cuda.empty_cache()
 
 
 # ------------------------------------------------------------------ a9 batched
