@@ -522,7 +522,14 @@ struct LaplaceBody {
 
     __device__ __forceinline__ Loop prologue(int64_t o, int, Step& st, bool, TeamShared&) const {
         st.i = o;
-        const int64_t i = 1 + o / (ny - 2), j = 1 + o % (ny - 2);
+        int64_t i, j;
+        if (o < ((int64_t)1 << 32) && ny - 2 < ((int64_t)1 << 32)) {   // 32-bit division when it fits
+            const uint32_t q = (uint32_t)o / (uint32_t)(ny - 2);
+            i = 1 + (int64_t)q;
+            j = 1 + (int64_t)((uint32_t)o - q * (uint32_t)(ny - 2));
+        } else {
+            i = 1 + o / (ny - 2), j = 1 + o % (ny - 2);
+        }
         return Loop{nx - 2, (i * ny + j) * nx + 1};
     }
     __device__ __forceinline__ void apply(const Loop& L, int64_t j) const {
