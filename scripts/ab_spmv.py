@@ -22,11 +22,16 @@ CFGS = {
     "S1 bv": dict(simdlen=1, threads_per_team=1024, blocked=True, vec128=True),
     "S2 b": dict(simdlen=2, threads_per_team=1024, blocked=True),
     "S1 cyc256": dict(simdlen=1, threads_per_team=256),
+    "S2 bv T768": dict(simdlen=2, threads_per_team=768, blocked=True, vec128=True),
+    "S1 bv T768": dict(simdlen=1, threads_per_team=768, blocked=True, vec128=True),
+    "S2 bv T512": dict(simdlen=2, threads_per_team=512, blocked=True, vec128=True),
 }
+if os.environ.get("AB_ONLY"):
+    CFGS = {k: v for k, v in CFGS.items() if k in os.environ["AB_ONLY"].split(",")}
 rounds = int(sys.argv[1]) if len(sys.argv) > 1 else 3
 res = {}
 for r in range(rounds):
-    for clean in ("0", "1"):
+    for clean in ("1",):
         os.environ["NEST_FLUSH_CLEAN"] = clean
         for name, cfg in CFGS.items():
             ts = []

@@ -176,8 +176,8 @@ __global__ void __launch_bounds__(1024, 2)
 // tuples l, l+S, ...  The first UNR iterations are issued as one predicated
 // block (all tuple loads, then all x gathers, then the FMAs in iteration
 // order -- same per-lane order as the plain loop), the rest in a plain loop.
-template <int S, int V, int UNR, int MINB, int XL = 0, bool RPF = false>
-__global__ void __launch_bounds__(1024, MINB)
+template <int S, int V, int UNR, int MINB, int XL = 0, bool RPF = false, int TB = 1024>
+__global__ void __launch_bounds__(TB, MINB)
     spmv2(const int64_t* __restrict__ rp, const int* __restrict__ col, const double* __restrict__ val,
           const double* __restrict__ x, double* __restrict__ y, int n, int chunk, int nnz, int64_t) {
     constexpr int LG = V == 2 ? 1 : 2;
@@ -363,13 +363,13 @@ int main(int argc, char** argv) {
         }
         CK(cudaDeviceSynchronize());
         const double alg = nnz * 12.0 + (n + 1) * 8.0 + n * 8.0 + n * 8.0;
-        const int T = 1024;
         const int G = 32;   // chunk granularity (a multiple of every variant's groups per warp)
         printf("# spmv n=%d nnz=%d far 1/%d alg %.3f GB\n", n, nnz, far_den, alg * 1e-9);
         struct V {
             const char* name;
             SpmvFn fn;
             int apw;   // 1: persisting access-policy window over x
+            int T = 1024;
         } vs[] = {
             {"base(nc/nc)", spmv<0, 0, false>, 0},
             {"x:L2last", spmv<1, 0, false>, 0},
@@ -398,6 +398,13 @@ int main(int argc, char** argv) {
             {"S2 V2 U2 rowptr prefetch", spmv2<2, 2, 2, 2, 0, true>, 2},
             {"S2 V2 U2 x:L1last rp-pf", spmv2<2, 2, 2, 2, 3, true>, 2},
             {"S2 V2 U2 (write-only flush)", spmv2<2, 2, 2, 2>, 0},
+            {"S2 V2 U3 T768x2", spmv2<2, 2, 3, 2, 0, false, 768>, 2, 768},
+            {"S2 V2 U2 T768x2", spmv2<2, 2, 2, 2, 0, false, 768>, 2, 768},
+            {"S2 V2 U4 T512x3", spmv2<2, 2, 4, 3, 0, false, 512>, 2, 512},
+            {"S2 V2 U3 T512x3", spmv2<2, 2, 3, 3, 0, false, 512>, 2, 512},
+            {"S2 V2 U2 T512x4", spmv2<2, 2, 2, 4, 0, false, 512>, 2, 512},
+            {"S4 V2 U2 T768x2", spmv2<4, 2, 2, 2, 0, false, 768>, 2, 768},
+            {"S1 V2 U4 T768x2", spmv2<1, 2, 4, 2, 0, false, 768>, 2, 768},
             {"S4 V2 U1", spmv2<4, 2, 1, 2>, 2},
             {"S4 V2 U2", spmv2<4, 2, 2, 2>, 2},
             {"S2 V4 U1", spmv2<2, 4, 1, 2>, 2},
@@ -428,6 +435,7 @@ int main(int argc, char** argv) {
                 CK(cudaStreamSetAttribute(st, cudaStreamAttributeAccessPolicyWindow, &a));
             }
             int nb = 0;
+            const int T = v.T;
             CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, v.fn, T, 0));
             const int grid = prop.multiProcessorCount * nb;
             int chunk = (n + grid - 1) / grid;
