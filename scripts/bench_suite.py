@@ -146,6 +146,76 @@ def g100(out):
     print("g100 done", flush=True)
 
 
+def cfg5(out):
+    """BASELINE configs[4] (100M x 100M, U{8..24} nnz/row, 1.6G nonzeros) on ONE GPU:
+    the headline and simdlen-1 configurations over the whole matrix, sampled
+    parity against the oracle, and a single-GPU emulation of the P-rank row
+    partition (each rank's rows as its own launch through the peer-gather
+    kernel, every x slice on this GPU: NVLink traffic is not exercised)."""
+    import numpy as np
+
+    import oracle  # test infrastructure: the checker (bench-side use, not the product path)
+    spec = R.CFG5
+    rp, col, val = R.spmv_matrix(spec)
+    x = R.spmv_x(spec)
+    nnz = int(val.size)
+    B = nnz * 12 + (spec.nrows + 1) * 8 + spec.nrows * 8 + spec.ncols * 8
+    t = [torch.from_numpy(a).cuda() for a in (rp, col, val, x)]
+    del col, val
+    y = torch.empty(spec.nrows, dtype=torch.float64, device="cuda")
+    res = []
+    for S, flags in ((2, "bv"), (4, "bv"), (8, "bv"), (2, "bq"), (4, "bq"), (1, "bv"), (1, "bq"), (2, "b"), (4, "b"),
+                     (1, "b"), (1, "")):
+        cfg = dict(simdlen=S, threads_per_team=1024 if "b" in flags else 256, blocked="b" in flags,
+                   vec128="v" in flags or "q" in flags, quad="q" in flags)
+        ms = timed(lambda: P.spmv_csr_f64(*t, y, **cfg), iters=5)
+        res.append(dict(cfg, ms=ms, GBs=B / ms / 1e6, frac_of_8TBs=B / ms / 1e6 / 8000.0))
+    # sampled parity of the headline configuration (R3 tolerance)
+    bcfg = {k: v for k, v in min(res, key=lambda r: r["ms"]).items() if k not in ("ms", "GBs", "frac_of_8TBs")}
+    P.spmv_csr_f64(*t, y, **bcfg)
+    yh = y.cpu().numpy()
+    rng = np.random.default_rng(5)
+    worst = 0.0
+    for s0 in np.concatenate([[0, spec.nrows - 64], rng.integers(0, spec.nrows - 64, 6)]):
+        rpl, cl, vl = R.spmv_matrix(spec, row_begin=int(s0), nrows=64)
+        yr, ar = oracle.spmv_csr_f64(rpl, cl, vl, x)
+        err = np.abs(yh[s0:s0 + 64] - yr)
+        assert np.all(err <= 1e-12 * ar), f"cfg5 parity at rows {s0}"
+        worst = max(worst, float(np.max(err / np.maximum(ar, 1e-300))))
+    # row partition emulated on one GPU: rank r's rows and CSR slice, x split in P slices
+    part = []
+    y_pairs = torch.empty_like(y)
+    best = min(res, key=lambda r: r["ms"])
+    hcfg = {k: best[k] for k in ("simdlen", "threads_per_team", "blocked", "vec128")}
+    P.spmv_csr_f64(*t, y_pairs, **hcfg)   # whole-matrix reference for the bitwise check (pairs)
+    for Pn in (2, 4, 8):
+        chunk = -(-spec.nrows // Pn)
+        xc = -(-spec.ncols // Pn)
+        xpad = torch.zeros(xc * Pn, dtype=torch.float64, device="cuda")
+        xpad[:spec.ncols] = t[3]
+        slices = [xpad[r * xc:(r + 1) * xc] for r in range(Pn)]
+        for r in (0, Pn - 1):
+            rb, re_ = r * chunk, min((r + 1) * chunk, spec.nrows)
+            k0, k1 = int(rp[rb]), int(rp[re_])
+            lrp = (t[0][rb:re_ + 1] - k0).contiguous()
+            lcol, lval = t[1][k0:k1].clone(), t[2][k0:k1].clone()
+            xp = P.XPeer(spec.ncols, nranks=Pn, rank=r, local_slices=slices)
+            yl = torch.empty(re_ - rb, dtype=torch.float64, device="cuda")
+            ms = timed(lambda: xp.spmv_csr_f64(spec.nrows, lrp, lcol, lval, yl, **hcfg), iters=5)
+            same = bool(torch.equal(yl, y_pairs[rb:re_]))
+            xp.close()
+            Br = (k1 - k0) * 12 + (re_ - rb + 1) * 8 + (re_ - rb) * 8 + spec.ncols * 8
+            part.append(dict(P=Pn, rank=r, rows=re_ - rb, nnz=k1 - k0, ms=ms, GBs=Br / ms / 1e6,
+                             bitwise_equal_whole=same))
+            del lrp, lcol, lval, yl
+        del xpad, slices
+    out["cfg5"] = dict(nnz=nnz, alg_bytes=B, results=res, best=min(res, key=lambda r: r["ms"]),
+                       parity_worst_rel_err=worst, partition_emulation=part)
+    del t
+    torch.cuda.empty_cache()
+    print("cfg5 done", json.dumps(out["cfg5"]["best"]), json.dumps(part), flush=True)
+
+
 def teams(out):
     """NEXT-1: the paper's two-level baseline (teams distribute in generic mode +
     parallel for) against the three-level path, CFG2 matrix."""
