@@ -22,6 +22,11 @@ for S in (2, 8, 32):
         P.spmv_csr_f64(rp, col, val, x, simdlen=S, mode=mode, x_halo=100)
         P.nested_stencil_f64(inp, coef, w, 4099, 8, simdlen=S, mode=mode)
         P.batched_matvec_f32(A, xb, 64, simdlen=S, mode=mode, outer_unroll=2)
+        P.batched_matvec_f32(A, xb, 64, simdlen=S, mode=mode)   # lean SPMD / generic drivers (U = 1)
+        P.spmv_csr_f64(rp, col, val, x, simdlen=S, mode=mode, blocked=True, vec128=True, threads_per_team=1024,
+                       team_chunk=64)
+        u = torch.rand(12 * 10 * 9, dtype=torch.float64, device="cuda")
+        P.laplace3d_f64(u, u.clone(), 12, 10, 9, 0.1, simdlen=S, mode=mode)
         P.probe_mapping(2, 37, simdlen=S, mode=mode)
 torch.cuda.synchronize()
 print("sanitize workload done")
