@@ -25,6 +25,11 @@ CFGS = {
     "S2 bv T768": dict(simdlen=2, threads_per_team=768, blocked=True, vec128=True),
     "S1 bv T768": dict(simdlen=1, threads_per_team=768, blocked=True, vec128=True),
     "S2 bv T512": dict(simdlen=2, threads_per_team=512, blocked=True, vec128=True),
+    "S2 v xwin4096 T1024": dict(simdlen=2, threads_per_team=1024, vec128=True, x_halo=4096),
+    "S2 v xwin3072 T1024": dict(simdlen=2, threads_per_team=1024, vec128=True, x_halo=3072),
+    "S2 v xwin4096 T512": dict(simdlen=2, threads_per_team=512, vec128=True, x_halo=4096),
+    "S4 v xwin4096 T1024": dict(simdlen=4, threads_per_team=1024, vec128=True, x_halo=4096),
+    "S1 v xwin4096 T1024": dict(simdlen=1, threads_per_team=1024, vec128=True, x_halo=4096),
 }
 if os.environ.get("AB_ONLY"):
     CFGS = {k: v for k, v in CFGS.items() if k in os.environ["AB_ONLY"].split(",")}

@@ -176,7 +176,7 @@ __global__ void __launch_bounds__(1024, 2)
 // tuples l, l+S, ...  The first UNR iterations are issued as one predicated
 // block (all tuple loads, then all x gathers, then the FMAs in iteration
 // order -- same per-lane order as the plain loop), the rest in a plain loop.
-template <int S, int V, int UNR, int MINB, int XL = 0, bool RPF = false, int TB = 1024>
+template <int S, int V, int UNR, int MINB, int XL = 0, bool RPF = false, int TB = 1024, int XS = 0>
 __global__ void __launch_bounds__(TB, MINB)
     spmv2(const int64_t* __restrict__ rp, const int* __restrict__ col, const double* __restrict__ val,
           const double* __restrict__ x, double* __restrict__ y, int n, int chunk, int nnz, int64_t) {
@@ -186,9 +186,23 @@ __global__ void __launch_bounds__(TB, MINB)
     const int cs = blockIdx.x * chunk;
     const int ce = min(n, cs + chunk);
     const unsigned mask = S == 32 ? 0xffffffffu : (((1u << S) - 1) << (S * ((threadIdx.x & 31) / S)));
+    extern __shared__ double xs[];   // XS: diagnostic -- gathers from an 8192-double shared window (wrong values)
+    if constexpr (XS) {
+        for (int k = threadIdx.x; k < 8192; k += blockDim.x) xs[k] = x[k];
+        __syncthreads();
+    }
     int nb = 0, ne = 0;
     if (RPF && cs + g < ce) nb = (int)__ldg(rp + cs + g), ne = (int)__ldg(rp + cs + g + 1);
-    for (int i = cs + g; i < ce; i += G) {
+    const int rounds = (ce - cs + G - 1) / G;
+    for (int k = 0; k < rounds; ++k) {
+        const int i = cs + g + k * G;
+        if constexpr (XS == 2) {
+            if (k % 4 == 0) __syncthreads();   // diag: a team barrier every 4 rows per group
+        }
+        if constexpr (XS == 3) {
+            if (k % 16 == 0) __syncthreads();
+        }
+        if (i >= ce) continue;
         int b, e;
         if constexpr (RPF) {
             b = nb, e = ne;
@@ -231,7 +245,8 @@ __global__ void __launch_bounds__(TB, MINB)
             const int k0 = ((b >> LG) + lane + u * S) << LG;
 #pragma unroll
             for (int q = 0; q < V; ++q)
-                xv[u][q] = (lane + u * S < trip && k0 + q >= b && k0 + q < e) ? ldx<XL>(x + c[u][q], 0) : 0.0;
+                xv[u][q] = (lane + u * S < trip && k0 + q >= b && k0 + q < e)
+                               ? (XS ? xs[c[u][q] & 8191] : ldx<XL>(x + c[u][q], 0)) : 0.0;
         }
 #pragma unroll
         for (int u = 0; u < UNR; ++u) {
@@ -399,6 +414,9 @@ int main(int argc, char** argv) {
             {"S2 V2 U2 x:L1last rp-pf", spmv2<2, 2, 2, 2, 3, true>, 2},
             {"S2 V2 U2 (write-only flush)", spmv2<2, 2, 2, 2>, 0},
             {"S2 V2 U3 T768x2", spmv2<2, 2, 3, 2, 0, false, 768>, 2, 768},
+            {"diag: S2 V2 U2, head gathers from smem", spmv2<2, 2, 2, 2, 0, false, 1024, 1>, 2, 1024},
+            {"diag: smem gathers + barrier every 4 rows", spmv2<2, 2, 2, 2, 0, false, 1024, 2>, 2, 1024},
+            {"diag: smem gathers + barrier every 16 rows", spmv2<2, 2, 2, 2, 0, false, 1024, 3>, 2, 1024},
             {"S2 V2 U2 T768x2", spmv2<2, 2, 2, 2, 0, false, 768>, 2, 768},
             {"S2 V2 U4 T512x3", spmv2<2, 2, 4, 3, 0, false, 512>, 2, 512},
             {"S2 V2 U3 T512x3", spmv2<2, 2, 3, 3, 0, false, 512>, 2, 512},
@@ -436,7 +454,9 @@ int main(int argc, char** argv) {
             }
             int nb = 0;
             const int T = v.T;
-            CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, v.fn, T, 0));
+            CK(cudaFuncSetAttribute(v.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, 65536));
+            const size_t dsm = strstr(v.name, "smem") ? 65536 : 0;
+            CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, v.fn, T, dsm));
             const int grid = prop.multiProcessorCount * nb;
             int chunk = (n + grid - 1) / grid;
             chunk = (chunk + G - 1) / G * G;
@@ -445,7 +465,7 @@ int main(int argc, char** argv) {
                 if (v.apw == 1) CK(cudaCtxResetPersistingL2Cache());
                 if (v.apw == 2) flush_wr(); else flush();
                 CK(cudaEventRecord(e0, st));
-                v.fn<<<grid, T, 0, st>>>(drp, dcol, dval, dx, dy, n, chunk, nnz, (int64_t)n * 8);
+                v.fn<<<grid, T, dsm, st>>>(drp, dcol, dval, dx, dy, n, chunk, nnz, (int64_t)n * 8);
                 CK(cudaEventRecord(e1, st));
                 CK(cudaEventSynchronize(e1));
                 float ms;
