@@ -123,7 +123,11 @@ struct FastDivU32 {
 struct XPeer {
     const double* const* slices;   // device array: nranks peer-mapped slice pointers
     FastDivU32 chunk;
+    const double* own;             // this rank's slice (columns [own_lo, own_lo + chunk.d))
+    uint32_t own_lo;
     __device__ __forceinline__ double operator()(int32_t c) const {
+        const uint32_t d = (uint32_t)c - own_lo;   // the banded columns of local rows: no owner lookup
+        if (d < chunk.d) return __ldg(own + d);
         const uint32_t o = chunk.div((uint32_t)c);
         const double* s = reinterpret_cast<const double*>(
             __ldg(reinterpret_cast<const unsigned long long*>(slices) + o));

@@ -22,6 +22,7 @@ struct nest_xpeer {
     bool local = false;                  // nest_xpeer_create_local: no IPC, no barrier
     bool opened = false;
     double* x_own = nullptr;             // this rank's slice (IPC mode, library-owned)
+    const double* own_slice = nullptr;   // this rank's slice as the kernel reads it (either form)
     uint64_t* flags_own = nullptr;       // barrier flags written by the peers (nranks)
     const double** d_slices = nullptr;   // device: nranks slice pointers
     uint64_t** d_peer_flags = nullptr;   // device: nranks pointers to each rank's flags
@@ -176,6 +177,7 @@ NEST_API nest_status nest_xpeer_create_local(int32_t nranks, int32_t rank, int64
     }
     xp->local = true;
     xp->opened = true;
+    xp->own_slice = slices[rank];
     *out = xp;
     return NEST_OK;
 }
@@ -238,7 +240,8 @@ NEST_API nest_status nest_spmv_csr_f64_xpeer(const nest_desc* desc, nest_xpeer* 
     // every rank's slice is written before anyone gathers from it
     if ((s = nest_xpeer_barrier(xp, stream)) != NEST_OK) return s;
     if (nrows_local > 0) {
-        const XPeer xa{xp->d_slices, FastDivU32::make((uint32_t)(xp->xchunk > 0 ? xp->xchunk : 1))};
+        const XPeer xa{xp->d_slices, FastDivU32::make((uint32_t)(xp->xchunk > 0 ? xp->xchunk : 1)),
+                       xp->local ? xp->own_slice : xp->x_own, (uint32_t)((int64_t)xp->rank * xp->xchunk)};
         if (vec) {
             s = launch_spmv_xpeer_vec(p, rowptr, colind, val, xa, y, fb, st, nnz);
         } else {
