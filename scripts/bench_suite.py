@@ -216,6 +216,41 @@ def cfg5(out):
     print("cfg5 done", json.dumps(out["cfg5"]["best"]), json.dumps(part), flush=True)
 
 
+def fig9(out):
+    """Fig 9 analogue: CSR SpMV time per simdlen and mode on the
+    short-row cfg2 matrix and its all-far variant, best variant per (S, mode)
+    among blocked teams of 1024 with scalar / 128-bit pair / quad loads."""
+    res = {}
+    for spec in (R.CFG2, R.CFG2_UNIFORM):
+        rp, col, val = R.spmv_matrix(spec)
+        x = R.spmv_x(spec)
+        t = [torch.from_numpy(a).cuda() for a in (rp, col, val, x)]
+        y = torch.empty(spec.nrows, dtype=torch.float64, device="cuda")
+        B = val.size * 12 + (spec.nrows + 1) * 8 + spec.nrows * 8 + spec.ncols * 8
+        rows = []
+        for S in (1, 2, 4, 8, 16, 32):
+            for mode in (("spmd",) if S == 1 else MODES):
+                best = None
+                for flags in ("b", "bv", "bq"):
+                    cfg = dict(simdlen=S, mode=mode, threads_per_team=1024, blocked=True, vec128=flags != "b",
+                               quad=flags == "bq")
+                    try:
+                        ms = timed(lambda: P.spmv_csr_f64(*t, y, **cfg), iters=5)
+                    except P.NestError:
+                        continue
+                    if best is None or ms < best["ms"]:
+                        best = dict(S=S, mode=mode, variant=flags, ms=ms, GBs=B / ms / 1e6)
+                rows.append(best)
+        s1 = rows[0]["ms"]
+        for r in rows:
+            r["speedup_vs_simdlen1"] = s1 / r["ms"]
+        res[spec.name] = dict(alg_bytes=B, results=rows)
+        del t
+        torch.cuda.empty_cache()
+    out["fig9"] = res
+    print("fig9 done", flush=True)
+
+
 def teams(out):
     """NEXT-1: the paper's two-level baseline (teams distribute in generic mode +
     parallel for) against the three-level path, CFG2 matrix."""
