@@ -23,6 +23,10 @@
 #ifndef NEST_VEC_UNROLL
 #define NEST_VEC_UNROLL 1
 #endif
+// float4 tuples per lane issued as one predicated block by the batched 128-bit body
+#ifndef NEST_BVEC_HEAD
+#define NEST_BVEC_HEAD -1   // -1: per simdlen (BatchedVecBody::head_for)
+#endif
 // tuples per lane issued as one predicated block by the 128-bit SpMV body
 #ifndef NEST_VEC_HEAD
 #define NEST_VEC_HEAD 2
@@ -431,6 +435,38 @@ struct BatchedVecBody {
         acc = Red<OP, float>::accum(acc, a.y, v.y);
         acc = Red<OP, float>::accum(acc, a.z, v.z);
         return Red<OP, float>::accum(acc, a.w, v.w);
+    }
+    // the lane's first head_for(S) float4 tuples as one predicated block (engine.cuh
+    // head_iters): every load in flight before the first fold; same fold order.
+    // Sized for the 64-wide rows of cfg4 (16 tuples: S = 4 -> the whole row);
+    // measured on cfg4 at U = 1: S = 4 5253 -> 6215 GB/s, S = 8 4614 -> 6084 GB/s.
+    static constexpr int head_for(int S) {
+        return NEST_BVEC_HEAD >= 0 ? NEST_BVEC_HEAD : (S == 1 || S == 4 ? 4 : S <= 8 ? 2 : 0);
+    }
+    template <int OP, int S>
+    __device__ __forceinline__ float accum_head(const Loop& L, int32_t id, float acc) const {
+        constexpr int H = head_for(S) > 0 ? head_for(S) : 1;
+        float4 a[H], v[H];
+#pragma unroll
+        for (int h = 0; h < H; ++h) {
+            const int32_t j = id + h * S;
+            if (j < L.trip) {
+                a[h] = __ldg(A + L.base + j);
+                v[h] = __ldg(x + L.xbase + j);
+            } else {
+                a[h] = v[h] = make_float4(0.f, 0.f, 0.f, 0.f);
+            }
+        }
+#pragma unroll
+        for (int h = 0; h < H; ++h) {
+            if (id + h * S < L.trip) {
+                acc = Red<OP, float>::accum(acc, a[h].x, v[h].x);
+                acc = Red<OP, float>::accum(acc, a[h].y, v[h].y);
+                acc = Red<OP, float>::accum(acc, a[h].z, v[h].z);
+                acc = Red<OP, float>::accum(acc, a[h].w, v[h].w);
+            }
+        }
+        return acc;
     }
     __device__ __forceinline__ void epilogue(const Step& st, float total) const { y[st.out] = total; }
 };

@@ -11,7 +11,7 @@ FL="-O3 -std=c++17 -gencode arch=compute_100a,code=sm_100a -lineinfo -Xcompiler 
 mkdir -p build_$name
 for f in paper_conf_icpp_wrightdtcc23_b200/csrc/*.cu; do
   b=$(basename $f .cu)
-  if grep -q "SpmvVecBody" $f || [ $b = spmv_vec2 ] || [ $b = spmv_vec4 ]; then
+  if grep -q "SpmvVecBody\|BatchedVecBody" $f || [ $b = spmv_vec2 ] || [ $b = spmv_vec4 ]; then
     nvcc $FL "$@" -c $f -o build_$name/$b.o &
   else
     cp build/$b.o build_$name/$b.o
@@ -21,3 +21,4 @@ wait
 nvcc -gencode arch=compute_100a,code=sm_100a -shared -cudart static -L$NCCL/lib -l:libnccl.so.2 \
      -Xlinker -rpath,$NCCL/lib -o build_$name/libnest.so build_$name/*.o
 echo built build_$name/libnest.so
+rm -f build_$name/*.o   # only the library travels to the GPU box
