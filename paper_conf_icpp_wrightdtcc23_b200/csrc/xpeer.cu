@@ -54,7 +54,15 @@ __global__ void xpeer_barrier_kernel(uint64_t* const* peer_flags, const uint64_t
     if (r < nranks) {
         __threadfence_system();
         st_release_sys(peer_flags[r] + rank, epoch);
-        while (ld_acquire_sys(my_flags + r) < epoch) __nanosleep(64);
+        // bounded wait: a peer that never arrives (lost process, broken mapping)
+        // traps after 120 s instead of hanging the stream forever
+        uint64_t t0, t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+        while (ld_acquire_sys(my_flags + r) < epoch) {
+            __nanosleep(64);
+            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+            if (t - t0 > 120000000000ull) __trap();
+        }
     }
     __syncthreads();
 }
