@@ -41,9 +41,11 @@
  *     rowptr monotone with rowptr[0] == 0 and rowptr[nrows] == nnz,
  *     0 <= colind < ncols; pointers suitably aligned for their type.
  *     nest_csr_validate() checks the CSR ones on the device.
- *   - The library allocates nothing per call.  Library-owned lazily-grown
- *     device scratch (the sharing-space global fallback)
- *     is released by nest_shutdown().
+ *   - The library allocates nothing per call in steady state.  Library-owned
+ *     lazily-grown device scratch (the sharing-space global fallback,
+ *     PAPER.md:680-684), one buffer per (device, stream) so that concurrent
+ *     launches on different streams never share slots, is released by
+ *     nest_shutdown() (all of the current device's buffers).
  */
 #ifndef NEST_H
 #define NEST_H

@@ -7,7 +7,9 @@
 #include <cstdint>
 #include <cstdarg>
 #include <cstdio>
+#include <map>
 #include <mutex>
+#include <utility>
 
 #include "internal.h"
 
@@ -227,16 +229,17 @@ struct Scratch {
     unsigned char* ptr = nullptr;
     size_t bytes = 0;
 };
+// One buffer per (device, stream): launches on different streams may run
+// concurrently and must not share slots; launches on one stream are ordered.
 static std::mutex g_scratch_mu;
-static Scratch g_scratch[64];
+static std::map<std::pair<int, void*>, Scratch> g_scratch;
 
-nest_status fallback_scratch(size_t bytes, unsigned char** out) {
+nest_status fallback_scratch(size_t bytes, unsigned char** out, void* stream) {
     int dev = 0;
     cudaError_t e = cudaGetDevice(&dev);
     if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
-    if (dev < 0 || dev >= 64) return fail(NEST_ERR_UNSUPPORTED, "device %d", dev);
     std::lock_guard<std::mutex> lk(g_scratch_mu);
-    Scratch& s = g_scratch[dev];
+    Scratch& s = g_scratch[std::make_pair(dev, stream)];
     if (s.bytes < bytes) {
         if (s.ptr) {
             e = cudaFree(s.ptr);   // synchronises: only on growth, never in steady state
@@ -255,11 +258,11 @@ nest_status fallback_scratch(size_t bytes, unsigned char** out) {
     return NEST_OK;
 }
 
-nest_status prepare_fallback(const Plan& p, unsigned char** fb) {
+nest_status prepare_fallback(const Plan& p, unsigned char** fb, void* stream) {
     *fb = nullptr;
     if (!p.fallback) return NEST_OK;
     const size_t bytes = (size_t)p.grid * (size_t)p.groups * (size_t)p.payload_bytes;
-    return fallback_scratch(bytes, fb);
+    return fallback_scratch(bytes, fb, stream);
 }
 
 // --------------------------------------------------------- device utilities
@@ -362,7 +365,7 @@ NEST_API nest_status nest_spmv_csr_f64(const nest_desc* desc, int64_t nrows, int
                     reinterpret_cast<uintptr_t>(x)) & 15))
         return fail(NEST_ERR_UNSUPPORTED, "NEST_F_STAGED needs 16-byte aligned colind, val and x");
     unsigned char* fb = nullptr;
-    if ((s = prepare_fallback(p, &fb)) != NEST_OK) return s;
+    if ((s = prepare_fallback(p, &fb, stream)) != NEST_OK) return s;
     if ((p.flags & NEST_F_VEC128) &&
         ((reinterpret_cast<uintptr_t>(val) & 15) ||
          (reinterpret_cast<uintptr_t>(colind) & ((p.flags & NEST_F_VEC_QUAD) ? 15 : 7))))
@@ -420,7 +423,7 @@ NEST_API nest_status nest_spmv_csr_f64_hostio(const nest_desc* desc, int64_t nro
     if (p.x_halo > 0 && (p.flags & NEST_F_VEC128) && (nnz >= ((int64_t)1 << 31) - 8 || nrows >= ((int64_t)1 << 31) - 8))
         return fail(NEST_ERR_UNSUPPORTED, "x_halo with NEST_F_VEC128 needs nnz, nrows < 2^31");
     unsigned char* fb = nullptr;
-    if ((s = prepare_fallback(p, &fb)) != NEST_OK) return s;
+    if ((s = prepare_fallback(p, &fb, stream)) != NEST_OK) return s;
     cudaStream_t st = as_stream(stream);
     cudaError_t e;
     if ((e = cudaMemcpyAsync(d_rowptr, h_rowptr, (size_t)(nrows + 1) * 8, cudaMemcpyHostToDevice, st)) ||
@@ -451,7 +454,7 @@ NEST_API nest_status nest_batched_matvec_f32(const nest_desc* desc, int64_t batc
         (n % 4 || (reinterpret_cast<uintptr_t>(A) & 15) || (reinterpret_cast<uintptr_t>(x) & 15)))
         return fail(NEST_ERR_UNSUPPORTED, "NEST_F_VEC128 (batched) needs n %% 4 == 0 and 16-byte aligned A and x");
     unsigned char* fb = nullptr;
-    if ((s = prepare_fallback(p, &fb)) != NEST_OK) return s;
+    if ((s = prepare_fallback(p, &fb, stream)) != NEST_OK) return s;
     return launch_batched(p, batch, m, n, A, x, y, fb, as_stream(stream));
 }
 
@@ -466,7 +469,7 @@ NEST_API nest_status nest_nested_stencil_f64(const nest_desc* desc, int64_t nout
     if (nouter == 0) return NEST_OK;
     if (!w || !out || (L > 0 && (!in || !coef))) return fail(NEST_ERR_INVALID_ARG, "in/coef/w/out is NULL");
     unsigned char* fb = nullptr;
-    if ((s = prepare_fallback(p, &fb)) != NEST_OK) return s;
+    if ((s = prepare_fallback(p, &fb, stream)) != NEST_OK) return s;
     return launch_stencil(p, nouter, L, in, coef, w, out, visits, fb, as_stream(stream));
 }
 
@@ -481,7 +484,7 @@ NEST_API nest_status nest_laplace3d_f64(const nest_desc* desc, int64_t nz, int64
     if (!u || !out) return fail(NEST_ERR_INVALID_ARG, "u/out is NULL");
     if (u == out) return fail(NEST_ERR_INVALID_ARG, "u and out must not alias (Jacobi step)");
     unsigned char* fb = nullptr;
-    if ((s = prepare_fallback(p, &fb)) != NEST_OK) return s;
+    if ((s = prepare_fallback(p, &fb, stream)) != NEST_OK) return s;
     return launch_laplace(p, nz, ny, nx, alpha, u, out, fb, as_stream(stream));
 }
 
@@ -497,7 +500,7 @@ NEST_API nest_status nest_probe_mapping(const nest_desc* desc, int32_t* out_map,
     nest_status s = make_plan(desc, outer, 1, probe_payload, &p);
     if (s != NEST_OK) return s;
     unsigned char* fb = nullptr;
-    if ((s = prepare_fallback(p, &fb)) != NEST_OK) return s;
+    if ((s = prepare_fallback(p, &fb, stream)) != NEST_OK) return s;
     return launch_probe(p, out_map, trip, hits, owner, totals, fb, as_stream(stream));
 }
 
@@ -529,10 +532,15 @@ NEST_API nest_status nest_shutdown(void) {
     cudaError_t e = cudaGetDevice(&dev);
     if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
     std::lock_guard<std::mutex> lk(g_scratch_mu);
-    if (dev >= 0 && dev < 64 && g_scratch[dev].ptr) {
-        e = cudaFree(g_scratch[dev].ptr);
-        g_scratch[dev] = Scratch{};
-        if (e != cudaSuccess) return cuda_fail(e, "cudaFree(fallback)");
+    cudaError_t first = cudaSuccess;
+    for (auto it = g_scratch.begin(); it != g_scratch.end();) {
+        if (it->first.first == dev) {
+            if (it->second.ptr && (e = cudaFree(it->second.ptr)) != cudaSuccess && first == cudaSuccess) first = e;
+            it = g_scratch.erase(it);
+        } else {
+            ++it;
+        }
     }
+    if (first != cudaSuccess) return cuda_fail(first, "cudaFree(fallback)");
     return NEST_OK;
 }

@@ -62,9 +62,9 @@ nest_status make_plan_fixed(const nest_desc* d, int64_t outer, int32_t steps_per
 
 // Library-owned global fallback for the sharing space:
 // grown lazily, never shrunk, released by nest_shutdown().
-nest_status fallback_scratch(size_t bytes, unsigned char** out);
+nest_status fallback_scratch(size_t bytes, unsigned char** out, void* stream);
 // the fallback a plan needs (nullptr when it needs none)
-nest_status prepare_fallback(const Plan& p, unsigned char** fb);
+nest_status prepare_fallback(const Plan& p, unsigned char** fb, void* stream);
 
 // Payload bytes a body posts per simd batch for a given unroll.
 int32_t spmv_payload(int32_t U);

@@ -185,7 +185,7 @@ NEST_API nest_status nest_region_program(const nest_desc* desc, const nest_regio
             fb_bytes += grid * G * payload;
     }
     unsigned char* fb = nullptr;
-    if (fb_bytes > 0 && (s = fallback_scratch((size_t)fb_bytes, &fb)) != NEST_OK) return s;
+    if (fb_bytes > 0 && (s = fallback_scratch((size_t)fb_bytes, &fb, stream)) != NEST_OK) return s;
     region_program_kernel<<<(unsigned)grid, T, smem, static_cast<cudaStream_t>(stream)>>>(prog, fb);
     const cudaError_t e = cudaGetLastError();
     return e == cudaSuccess ? NEST_OK : cuda_fail(e, "region program launch");

@@ -243,7 +243,7 @@ NEST_API nest_status nest_spmv_csr_f64_xpeer(const nest_desc* desc, nest_xpeer* 
     if (vec && ((reinterpret_cast<uintptr_t>(val) & 15) || (reinterpret_cast<uintptr_t>(colind) & 7)))
         return fail(NEST_ERR_UNSUPPORTED, "NEST_F_VEC128 needs 16-byte aligned val and 8-byte aligned colind");
     unsigned char* fb = nullptr;
-    if ((s = prepare_fallback(p, &fb)) != NEST_OK) return s;
+    if ((s = prepare_fallback(p, &fb, stream)) != NEST_OK) return s;
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     // every rank's slice is written before anyone gathers from it
     if ((s = nest_xpeer_barrier(xp, stream)) != NEST_OK) return s;
