@@ -171,6 +171,27 @@ def test_spmv_zero_nnz_and_zero_rows(P):
     assert y0.numel() == 0
 
 
+def test_fallback_concurrent_streams(P, banded):
+    """Generic-SMEM launches whose payload exceeds the slot use the library's global
+    fallback; two of them in flight on different streams must not
+    share slots (one scratch buffer per stream)."""
+    rp, col, val, x, yref, aref = banded["int"]
+    t = [dev(rp), dev(col), dev(val), dev(x)]
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    torch.cuda.synchronize()
+    ys = []
+    for _ in range(4):
+        for st in (s1, s2):
+            y = torch.empty(rp.size - 1, dtype=torch.float64, device="cuda")
+            P.spmv_csr_f64(*t, y, simdlen=2, mode="generic_smem", sharing_bytes=64, stream=st)
+            ys.append(y)
+    torch.cuda.synchronize()
+    info = P.plan(rp.size - 1, 24, simdlen=2, mode="generic_smem", sharing_bytes=64)
+    assert info["uses_global_fallback"] == 1
+    for y in ys:
+        assert np.array_equal(bits(host(y)), bits(yref))
+
+
 def test_csr_validate(P, cfg1):
     rp, col, val, x, _, _ = cfg1["real"]
     assert P.csr_validate(dev(rp), dev(col), 1024) == 0
