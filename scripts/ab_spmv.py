@@ -30,6 +30,9 @@ CFGS = {
     "S2 v xwin4096 T512": dict(simdlen=2, threads_per_team=512, vec128=True, x_halo=4096),
     "S4 v xwin4096 T1024": dict(simdlen=4, threads_per_team=1024, vec128=True, x_halo=4096),
     "S1 v xwin4096 T1024": dict(simdlen=1, threads_per_team=1024, vec128=True, x_halo=4096),
+    "S2 v xwin4096 U2": dict(simdlen=2, threads_per_team=1024, vec128=True, x_halo=4096, outer_unroll=2),
+    "S2 v xwin4096 U4": dict(simdlen=2, threads_per_team=1024, vec128=True, x_halo=4096, outer_unroll=4),
+    "S4 v xwin4096 U2": dict(simdlen=4, threads_per_team=1024, vec128=True, x_halo=4096, outer_unroll=2),
 }
 if os.environ.get("AB_ONLY"):
     CFGS = {k: v for k, v in CFGS.items() if k in os.environ["AB_ONLY"].split(",")}

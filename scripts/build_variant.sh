@@ -2,7 +2,7 @@
 # Build a variant of libnest.so with extra nvcc defines into build_<name>/ (A/B
 # experiments on the GPU box: copy it over paper_conf_icpp_wrightdtcc23_b200/libnest.so).
 # Only the SpMV tuple-body translation units are recompiled; the rest come from build/.
-# usage: scripts/build_variant.sh h0 -DNEST_VEC_HEAD=0
+# usage: scripts/build_variant.sh h0 -DNEST_VEC_HEAD=0   (VARIANT_ALL=1: recompile every unit)
 set -e
 name=$1; shift
 cd "$(dirname "$0")/.."
@@ -11,7 +11,7 @@ FL="-O3 -std=c++17 -gencode arch=compute_100a,code=sm_100a -lineinfo -Xcompiler 
 mkdir -p build_$name
 for f in paper_conf_icpp_wrightdtcc23_b200/csrc/*.cu; do
   b=$(basename $f .cu)
-  if grep -q "SpmvVecBody\|BatchedVecBody\|StencilBody" $f || [ $b = spmv_vec2 ] || [ $b = spmv_vec4 ]; then
+  if [ -n "$VARIANT_ALL" ] || grep -q "SpmvVecBody\|BatchedVecBody\|StencilBody" $f || [ $b = spmv_vec2 ] || [ $b = spmv_vec4 ]; then
     nvcc $FL "$@" -c $f -o build_$name/$b.o &
   else
     cp build/$b.o build_$name/$b.o
