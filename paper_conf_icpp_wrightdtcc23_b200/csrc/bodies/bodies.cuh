@@ -24,6 +24,9 @@
 #define NEST_VEC_UNROLL 1
 #endif
 // float4 tuples per lane issued as one predicated block by the batched 128-bit body
+#ifndef NEST_SCALAR_HEAD
+#define NEST_SCALAR_HEAD -1   // -1: per simdlen (SpmvBody::head_for); 0: none
+#endif
 #ifndef NEST_BVEC_HEAD
 #define NEST_BVEC_HEAD -1   // -1: per simdlen (BatchedVecBody::head_for)
 #endif
@@ -212,6 +215,31 @@ struct SpmvBody {
         const int32_t c = HINTS ? ld_stream(col + k) : __ldg(col + k);
         const double v = HINTS ? ld_stream(val + k) : __ldg(val + k);
         return Red<OP, double>::accum(acc, v, x(c));
+    }
+    // the lane's first head_for(S) nonzeros (j = id, id + S, ...) as one predicated
+    // block: every colind/val load, then every x gather, then the folds in order
+    // (engine.cuh head_iters; same per-lane order, bit-identical)
+    static constexpr int head_for(int S) {
+        return NEST_SCALAR_HEAD >= 0 ? NEST_SCALAR_HEAD : (S <= 8 ? 2 : 1);   // 4 at S <= 2 needs 40 registers
+    }
+    template <int OP, int S>
+    __device__ __forceinline__ double accum_head(const Loop& L, int32_t id, double acc) const {
+        constexpr int H = head_for(S) > 0 ? head_for(S) : 1;
+        int32_t c[H];
+        double v[H], xv[H];
+#pragma unroll
+        for (int h = 0; h < H; ++h) {
+            const I j = (I)id + (I)(h * S);
+            const I k = L.base + j;
+            c[h] = j < L.trip ? (HINTS ? ld_stream(col + k) : __ldg(col + k)) : 0;
+            v[h] = j < L.trip ? (HINTS ? ld_stream(val + k) : __ldg(val + k)) : 0.0;
+        }
+#pragma unroll
+        for (int h = 0; h < H; ++h) xv[h] = (I)id + (I)(h * S) < L.trip ? x(c[h]) : 0.0;
+#pragma unroll
+        for (int h = 0; h < H; ++h)
+            if ((I)id + (I)(h * S) < L.trip) acc = Red<OP, double>::accum(acc, v[h], xv[h]);
+        return acc;
     }
     __device__ __forceinline__ void epilogue(const Step& st, double total) const { y[st.i] = total; }
 };

@@ -30,6 +30,12 @@ CFGS = {
     "S2 v xwin4096 T512": dict(simdlen=2, threads_per_team=512, vec128=True, x_halo=4096),
     "S4 v xwin4096 T1024": dict(simdlen=4, threads_per_team=1024, vec128=True, x_halo=4096),
     "S1 v xwin4096 T1024": dict(simdlen=1, threads_per_team=1024, vec128=True, x_halo=4096),
+    "S2 b gsmem": dict(simdlen=2, mode="generic_smem", threads_per_team=1024, blocked=True),
+    "S2 b gshfl": dict(simdlen=2, mode="generic_shfl", threads_per_team=1024, blocked=True),
+    "S4 b": dict(simdlen=4, threads_per_team=1024, blocked=True),
+    "S8 b": dict(simdlen=8, threads_per_team=1024, blocked=True),
+    "S8 b gsmem": dict(simdlen=8, mode="generic_smem", threads_per_team=1024, blocked=True),
+    "S1 b": dict(simdlen=1, threads_per_team=1024, blocked=True),
     "S2 v xwin4096 U2": dict(simdlen=2, threads_per_team=1024, vec128=True, x_halo=4096, outer_unroll=2),
     "S2 v xwin4096 U4": dict(simdlen=2, threads_per_team=1024, vec128=True, x_halo=4096, outer_unroll=4),
     "S4 v xwin4096 U2": dict(simdlen=4, threads_per_team=1024, vec128=True, x_halo=4096, outer_unroll=2),
