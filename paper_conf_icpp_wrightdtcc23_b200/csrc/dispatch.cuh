@@ -11,12 +11,19 @@
 namespace nest {
 
 template <class Body, int U, int S, int MODE, int OP>
+constexpr auto kernel_of() {
+    if constexpr (U == 1 && two_teams_per_sm<Body>::value) return nest_kernel_2pm<S, MODE, OP, U, Body>;
+    else return nest_kernel<S, MODE, OP, U, Body>;
+}
+
+template <class Body, int U, int S, int MODE, int OP>
 nest_status launch_one(const Plan& p, const Body& body, unsigned char* fb, cudaStream_t st) {
+    constexpr auto kern = kernel_of<Body, U, S, MODE, OP>();
     // a team size the instantiation cannot run (registers) is reported before launching
     static int max_threads = 0;
     if (max_threads == 0) {
         cudaFuncAttributes fa;
-        if (cudaFuncGetAttributes(&fa, nest_kernel<S, MODE, OP, U, Body>) == cudaSuccess)
+        if (cudaFuncGetAttributes(&fa, kern) == cudaSuccess)
             max_threads = fa.maxThreadsPerBlock;
         else
             cudaGetLastError();
@@ -26,11 +33,11 @@ nest_status launch_one(const Plan& p, const Body& body, unsigned char* fb, cudaS
                     "threads_per_team %d exceeds this variant's limit of %d (registers); use a smaller team or "
                     "outer_unroll", p.block, max_threads);
     if (p.smem_bytes > 48 * 1024) {
-        const cudaError_t e = cudaFuncSetAttribute(nest_kernel<S, MODE, OP, U, Body>,
+        const cudaError_t e = cudaFuncSetAttribute(kern,
                                                    cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem_bytes);
         if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(max dynamic smem)");
     }
-    nest_kernel<S, MODE, OP, U, Body><<<p.grid, p.block, p.smem_bytes, st>>>(
+    kern<<<p.grid, p.block, p.smem_bytes, st>>>(
         body, p.outer, p.slot_bytes, fb, (p.flags & NEST_F_BLOCKED) ? p.chunk : 0, p.pipe_off);
     const cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e, "kernel launch");
