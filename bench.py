@@ -294,8 +294,9 @@ def run_gpu(args, rank, world, local_rank):
 
         body = ("SpmvVecBody<0,4>" if "q" in best[5] else "SpmvVecBody<0,2>" if "v" in best[5]
                 else f"SpmvBody<{int('h' in best[5])},0>")
+        kname = "nest_kernel_2pm" if ("v" in best[5] or "q" in best[5]) and best[2] == 1 else "nest_kernel"
         kernel_name = (f"spmv_staged_kernel<S={best[0]},{best[1]},SUM,U={best[2]}>" if "s" in best[5] else
-                       f"nest_kernel<S={best[0]},{best[1]},SUM,U={best[2]},{body}>")
+                       f"{kname}<S={best[0]},{best[1]},SUM,U={best[2]},{body}>")
         traffic = None
         try:
             with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
@@ -421,7 +422,7 @@ def run_gpu(args, rank, world, local_rank):
         per_gpu = line["value"] / world
         line["roofline"] = {"bound": "hbm", "achieved": per_gpu, "peak": peak, "unit": "GB/s",
                             "frac": per_gpu / peak, "traffic": None, "peak_source": peak_src,
-                            "kernel": f"nest_kernel<S={cfg['simdlen']},{cfg['mode']},SUM,U=1,SpmvVecBody<0,2,int,"
+                            "kernel": f"nest_kernel_2pm<S={cfg['simdlen']},{cfg['mode']},SUM,U=1,SpmvVecBody<0,2,int,"
                                       f"{'XPeer' if head == 'xpeer' else 'XLocal'}>>",
                             "note": "per GPU: algorithmic bytes of all ranks / world / max-over-ranks step time"}
         print(json.dumps(line), flush=True)
