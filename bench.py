@@ -294,7 +294,8 @@ def run_gpu(args, rank, world, local_rank):
 
         body = ("SpmvVecBody<0,4>" if "q" in best[5] else "SpmvVecBody<0,2>" if "v" in best[5]
                 else f"SpmvBody<{int('h' in best[5])},0>")
-        kname = "nest_kernel_2pm" if ("v" in best[5] or "q" in best[5]) and best[2] == 1 else "nest_kernel"
+        kname = ("nest_kernel_2pm" if ("v" in best[5] or "q" in best[5]) and best[2] == 1
+                 and not ("q" in best[5] and best[0] == 1) else "nest_kernel")
         kernel_name = (f"spmv_staged_kernel<S={best[0]},{best[1]},SUM,U={best[2]}>" if "s" in best[5] else
                        f"{kname}<S={best[0]},{best[1]},SUM,U={best[2]},{body}>")
         traffic = None

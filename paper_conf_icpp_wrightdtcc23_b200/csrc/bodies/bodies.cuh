@@ -260,7 +260,9 @@ struct SpmvVecBody {
     // fewer registers, so two teams of 1024 fit an SM)
     using Acc = double;
     using OuterIndex = I;   // launcher: I = int32_t only when spmv_index32()
-    static constexpr bool kTwoTeamsPerSm = true;   // engine.cuh two_teams_per_sm (U = 1)
+    // engine.cuh two_teams_per_sm (U = 1): cap registers at 32 for two teams of 1024
+    // per SM -- except quads at simdlen 1, which would spill (measured slower)
+    static constexpr bool two_teams_for(int S) { return !(V == 4 && S == 1); }
     static constexpr int kLoopUnroll = NEST_VEC_UNROLL;   // V nonzeros per iteration already
     struct Loop {
         I base;         // rowptr[i]

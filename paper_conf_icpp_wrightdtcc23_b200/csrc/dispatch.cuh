@@ -12,7 +12,7 @@ namespace nest {
 
 template <class Body, int U, int S, int MODE, int OP>
 constexpr auto kernel_of() {
-    if constexpr (U == 1 && two_teams_per_sm<Body>::value) return nest_kernel_2pm<S, MODE, OP, U, Body>;
+    if constexpr (U == 1 && two_teams_per_sm<Body, S>::value) return nest_kernel_2pm<S, MODE, OP, U, Body>;
     else return nest_kernel<S, MODE, OP, U, Body>;
 }
 
