@@ -171,7 +171,24 @@ def g100(out):
                                           blocked=blocked, vec128=vec), iters=10)
         res.append(dict(S=S, mode=mode, U=U, T=T, blocked=blocked, vec128=vec, ms=ms, GBs=B / ms / 1e6,
                         frac_of_8TBs=B / ms / 1e6 / 8000.0))
-    out["g100"] = dict(nnz=int(val.size), alg_bytes=B, results=res, best=min(res, key=lambda r: r["ms"]))
+    # warm-x variant: L2 flushed, then x read once (x.sum()) before each timed launch
+    best = min(res, key=lambda r: r["ms"])
+    bcfg = dict(simdlen=best["S"], mode=best["mode"], outer_unroll=best["U"], threads_per_team=best["T"],
+                blocked=best["blocked"], vec128=best["vec128"])
+    ts = []
+    for _ in range(10):
+        P.l2_flush(flush)
+        t[3].sum()
+        e0, e1 = torch.cuda.Event(True), torch.cuda.Event(True)
+        e0.record()
+        P.spmv_csr_f64(*t, y, **bcfg)
+        e1.record()
+        e1.synchronize()
+        ts.append(e0.elapsed_time(e1))
+    wms = statistics.median(ts)
+    warm = dict(bcfg, ms=wms, GBs=B / wms / 1e6, note="x read into L2 before each launch (x is 100 MB: "
+                "beyond the ~72-80 MB effective L2 for gathers, so only partly resident)")
+    out["g100"] = dict(nnz=int(val.size), alg_bytes=B, results=res, best=best, warm_x=warm)
     print("g100 done", flush=True)
 
 
