@@ -120,7 +120,22 @@ def cpu_baseline(spec, min_seconds=10.0, max_seconds=30.0):
         passes += 1
     return {"value": B * passes / t_total / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
             "sample": f"{passes} full passes of {spec.name} ({spec.nrows} rows, {val.size} nnz), "
-                      f"{t_total:.1f} s single-threaded C (oracle/oracle.c)"}
+                      f"{t_total:.1f} s single-threaded C (oracle/oracle.c)",
+            "host": host_cpu()}
+
+
+def host_cpu():
+    """The box's CPU model and logical core count (context for cpu_baseline)."""
+    model = "unknown"
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    model = line.split(":", 1)[1].strip()
+                    break
+    except OSError:
+        pass
+    return {"model": model, "logical_cores": os.cpu_count()}
 
 
 def run_reference(args, rank, world):
@@ -148,7 +163,7 @@ def run_reference(args, rank, world):
                                    f"U{{{spec.nnz_min}..{spec.nnz_max}}} banded+far (W={spec.band_w}, "
                                    f"far 1/{spec.far_den})", "nnz": int(val.size), "alg_bytes": B},
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
-                             "sample": f"the full {spec.name} matrix per step, single-threaded C oracle"},
+                             "sample": f"the full {spec.name} matrix per step, single-threaded C oracle", "host": host_cpu()},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
