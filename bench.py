@@ -343,7 +343,12 @@ def run_gpu(args, rank, world, local_rank):
                          "traffic_over_alg_bytes": (traffic / B) if traffic else None,
                          "kernel": kernel_name, "frac_of_8TBs_spec": value / 8000.0},
             "e2e": {"value": B / (ms_e2e / 1e3) / 1e9, "unit": UNIT, "h2d_bytes_per_step": h2d,
-                    "d2h_bytes_per_step": d2h, "ms_per_step": ms_e2e},
+                    "d2h_bytes_per_step": d2h, "ms_per_step": ms_e2e,
+                    "h2d_gbs": h2d / (ms_e2e / 1e3) / 1e9,
+                    "pipeline": (f"{int(os.environ['NEST_HOSTIO_CHUNKS'])} row chunks (forced)"
+                                 if os.environ.get("NEST_HOSTIO_CHUNKS") else
+                                 f"{min(32, max(1, -(-nnz // (8 << 20))))} row chunks of ~8 Mi nonzeros")
+                    + ": chunk c's SpMV and y copy overlap the H2D of chunks > c"},
             "gpu_launches": 3 * args.steps,
             "gpu_launches_detail": "per step: 1 SpMV kernel + 2 l2 flush kernels (write, clean-read; outside the step events)",
             "clocks": clk.summary(),

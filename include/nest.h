@@ -178,8 +178,18 @@ nest_status nest_spmv_csr_f64(const nest_desc *desc, int64_t nrows, int64_t ncol
 
 /* a8 end to end from HOST buffers (pinned for asynchronous copies): copies
  * rowptr/colind/val/x into `d_workspace` (device, >= nest_spmv_hostio_workspace_bytes),
- * runs nest_spmv_csr_f64 and copies y back into h_y, all on `stream`.  The
- * host buffers must stay valid until the stream reaches that point. */
+ * runs nest_spmv_csr_f64 and copies y back into h_y.  Above 8 Mi nonzeros the
+ * rows are split into chunks of ~8 Mi nonzeros (at most 32; NEST_HOSTIO_CHUNKS
+ * overrides): x, then each chunk's rowptr/colind/val cross on a library-owned
+ * H2D stream, chunk c's SpMV runs on `stream` once the entries it can read
+ * have landed, and its y rows return on a library-owned D2H stream, so the
+ * copies overlap the kernels and the two PCIe directions overlap each other.
+ * Ordering is still that of `stream`: the copies start after the work queued
+ * on it before the call, and work queued on it after the call starts after
+ * the last y row is on the host.  Results equal nest_spmv_csr_f64's bit for
+ * bit.  rowptr must start at 0 and end at nnz.  The host buffers must stay
+ * valid, and h_y unread, until `stream` reaches that point.  Staged and
+ * x_halo variants copy in one shot. */
 size_t nest_spmv_hostio_workspace_bytes(int64_t nrows, int64_t ncols, int64_t nnz);
 nest_status nest_spmv_csr_f64_hostio(const nest_desc *desc, int64_t nrows, int64_t ncols,
                                      int64_t nnz, const int64_t *h_rowptr,

@@ -3,6 +3,7 @@
 #include <cstdlib>
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <climits>
 #include <cstdint>
 #include <cstdarg>
@@ -390,6 +391,139 @@ NEST_API size_t nest_spmv_hostio_workspace_bytes(int64_t nrows, int64_t ncols, i
            align256((size_t)ncols * 8) + align256((size_t)nrows * 8);
 }
 
+// ---------------------------------------- a8 end to end: chunked pipeline
+// The host->device copy of the matrix is the bound of the end-to-end call
+// (PCIe, ~50 GB/s against ~4 TB/s for the SpMV itself).  Rows are split into
+// chunks of about kHostioChunkNnz nonzeros: x first, then per chunk its rowptr
+// slice, colind and val on an H2D stream; chunk c's SpMV runs on the caller's
+// stream once the copies it reads have landed, and its y rows go back on a
+// D2H stream while later chunks are still crossing the bus (the two PCIe
+// directions are independent).  Same kernel, same per-row arithmetic as the
+// single-shot path: results are bit-identical.
+static constexpr int64_t kHostioChunkNnz = int64_t(8) << 20;
+static constexpr int kHostioMaxChunks = 32;
+
+static int hostio_chunks(int64_t nnz) {
+    static const int forced = [] {
+        const char* e = std::getenv("NEST_HOSTIO_CHUNKS");   // A/B experiments (1 = single shot)
+        return e ? std::atoi(e) : 0;
+    }();
+    int64_t k = forced > 0 ? forced : (nnz + kHostioChunkNnz - 1) / kHostioChunkNnz;
+    if (k < 1) k = 1;
+    if (k > kHostioMaxChunks) k = kHostioMaxChunks;
+    return (int)k;
+}
+
+struct HostioStreams {
+    cudaStream_t h2d = nullptr, d2h = nullptr;
+    cudaEvent_t ev[2 * kHostioMaxChunks + 2] = {};
+};
+static std::mutex g_hostio_mu;
+static std::map<int, HostioStreams> g_hostio;
+
+static void hostio_destroy(HostioStreams& h) {
+    for (cudaEvent_t& ev : h.ev)
+        if (ev) cudaEventDestroy(ev), ev = nullptr;
+    if (h.h2d) cudaStreamDestroy(h.h2d), h.h2d = nullptr;
+    if (h.d2h) cudaStreamDestroy(h.d2h), h.d2h = nullptr;
+}
+
+// caller holds g_hostio_mu
+static nest_status hostio_streams(HostioStreams** out) {
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
+    auto it = g_hostio.find(dev);
+    if (it == g_hostio.end()) {
+        HostioStreams h;
+        if ((e = cudaStreamCreateWithFlags(&h.h2d, cudaStreamNonBlocking)) == cudaSuccess)
+            e = cudaStreamCreateWithFlags(&h.d2h, cudaStreamNonBlocking);
+        for (cudaEvent_t& ev : h.ev)
+            if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ev, cudaEventDisableTiming);
+        if (e != cudaSuccess) {
+            hostio_destroy(h);
+            return cuda_fail(e, "hostio streams/events");
+        }
+        it = g_hostio.emplace(dev, h).first;
+    }
+    *out = &it->second;
+    return NEST_OK;
+}
+
+static nest_status spmv_hostio_pipelined(const nest_desc* desc, int nchunks, int64_t nrows,
+                                         int64_t ncols, int64_t nnz, const int64_t* h_rowptr,
+                                         const int32_t* h_colind, const double* h_val, const double* h_x,
+                                         double* h_y, int64_t* d_rowptr, int32_t* d_col, double* d_val,
+                                         double* d_x, double* d_y, unsigned char* fb, cudaStream_t st) {
+    // chunk c = rows [r[c], r[c+1]) with nonzeros [h_rowptr[r[c]], h_rowptr[r[c+1]]);
+    // boundaries at the rows where the nonzero count crosses c * nnz / nchunks
+    int64_t r[kHostioMaxChunks + 1];
+    r[0] = 0;
+    for (int c = 1; c < nchunks; ++c) {
+        const int64_t target = h_rowptr[0] + (nnz * c) / nchunks;
+        int64_t lo = r[c - 1], hi = nrows;   // first row whose start >= target
+        while (lo < hi) {
+            const int64_t mid = lo + (hi - lo) / 2;
+            if (h_rowptr[mid] < target) lo = mid + 1; else hi = mid;
+        }
+        r[c] = lo;
+    }
+    r[nchunks] = nrows;
+    std::lock_guard<std::mutex> lk(g_hostio_mu);
+    HostioStreams* h = nullptr;
+    nest_status s = hostio_streams(&h);
+    if (s != NEST_OK) return s;
+    cudaEvent_t ev_start = h->ev[0], ev_done = h->ev[1];
+    cudaEvent_t* ev_in = h->ev + 2;
+    cudaEvent_t* ev_k = h->ev + 2 + kHostioMaxChunks;
+    cudaError_t e;
+    // everything earlier on the caller's stream (a previous call reading this workspace) first
+    if ((e = cudaEventRecord(ev_start, st)) || (e = cudaStreamWaitEvent(h->h2d, ev_start, 0)) ||
+        (e = cudaStreamWaitEvent(h->d2h, ev_start, 0)))
+        return cuda_fail(e, "hostio start");
+    if (ncols && (e = cudaMemcpyAsync(d_x, h_x, (size_t)ncols * 8, cudaMemcpyHostToDevice, h->h2d)))
+        return cuda_fail(e, "host->device copy (x)");
+    int64_t zb[kHostioMaxChunks + 1];   // nonzero boundaries, relative to the arrays
+    for (int c = 0; c <= nchunks; ++c) zb[c] = h_rowptr[r[c]];
+    for (int c = 0; c < nchunks; ++c) {
+        // rowptr entries [r[c] + (c > 0), r[c+1]]: disjoint slices, chunk c's bounds all covered by copies <= c
+        const int64_t p0r = r[c] + (c > 0), p1r = r[c + 1];
+        if (p1r >= p0r && (e = cudaMemcpyAsync(d_rowptr + p0r, h_rowptr + p0r, (size_t)(p1r - p0r + 1) * 8,
+                                               cudaMemcpyHostToDevice, h->h2d)))
+            return cuda_fail(e, "host->device copy (rowptr)");
+        const int64_t z0 = zb[c], z1 = zb[c + 1];
+        if (z1 > z0 &&
+            ((e = cudaMemcpyAsync(d_col + z0, h_colind + z0, (size_t)(z1 - z0) * 4, cudaMemcpyHostToDevice, h->h2d)) ||
+             (e = cudaMemcpyAsync(d_val + z0, h_val + z0, (size_t)(z1 - z0) * 8, cudaMemcpyHostToDevice, h->h2d))))
+            return cuda_fail(e, "host->device copy (colind/val)");
+        if ((e = cudaEventRecord(ev_in[c], h->h2d))) return cuda_fail(e, "hostio event");
+    }
+    for (int c = 0; c < nchunks; ++c) {
+        const int64_t rows = r[c + 1] - r[c];
+        // 128-bit tuples read up to 3 entries past the chunk's last nonzero (unused):
+        // wait for the copy that holds the last entry the chunk can touch
+        const int64_t last = std::min<int64_t>(nnz, (zb[c + 1] + 3) & ~(int64_t)3) - 1;
+        int j = c;
+        while (j + 1 < nchunks && zb[j + 1] <= last) ++j;
+        if ((e = cudaStreamWaitEvent(st, ev_in[j], 0))) return cuda_fail(e, "hostio wait");
+        if (rows > 0) {
+            Plan p;
+            if ((s = make_plan(desc, rows, 1, spmv_payload, &p, true)) != NEST_OK) return s;
+            if ((s = launch_spmv(p, (p.flags & NEST_F_STREAM_HINTS) != 0, rows, d_rowptr + r[c], d_col, d_val,
+                                 d_x, d_y + r[c], fb, st, nnz)) != NEST_OK)
+                return s;
+        }
+        if ((e = cudaEventRecord(ev_k[c], st)) || (e = cudaStreamWaitEvent(h->d2h, ev_k[c], 0)))
+            return cuda_fail(e, "hostio event");
+        if (rows > 0 && (e = cudaMemcpyAsync(h_y + r[c], d_y + r[c], (size_t)rows * 8, cudaMemcpyDeviceToHost, h->d2h)))
+            return cuda_fail(e, "device->host copy");
+    }
+    // the caller's stream completes only after the last y rows are on the host
+    if ((e = cudaEventRecord(ev_done, h->d2h)) || (e = cudaStreamWaitEvent(st, ev_done, 0)))
+        return cuda_fail(e, "hostio done");
+    return NEST_OK;
+}
+
 NEST_API nest_status nest_spmv_csr_f64_hostio(const nest_desc* desc, int64_t nrows, int64_t ncols,
                                               int64_t nnz, const int64_t* h_rowptr,
                                               const int32_t* h_colind, const double* h_val,
@@ -407,6 +541,9 @@ NEST_API nest_status nest_spmv_csr_f64_hostio(const nest_desc* desc, int64_t nro
         return fail(NEST_ERR_INVALID_ARG, "workspace %zu bytes < %zu", workspace_bytes, need);
     if (!h_rowptr || !h_y || (nnz > 0 && (!h_colind || !h_val || !h_x)))
         return fail(NEST_ERR_INVALID_ARG, "host buffer is NULL");
+    if (h_rowptr[0] != 0 || h_rowptr[nrows] != nnz)
+        return fail(NEST_ERR_INVALID_ARG, "rowptr must run from 0 to nnz (%lld .. %lld, nnz %lld)",
+                    (long long)h_rowptr[0], (long long)h_rowptr[nrows], (long long)nnz);
     unsigned char* w = static_cast<unsigned char*>(d_workspace);
     int64_t* d_rowptr = reinterpret_cast<int64_t*>(w);
     w += align256((size_t)(nrows + 1) * 8);
@@ -426,6 +563,10 @@ NEST_API nest_status nest_spmv_csr_f64_hostio(const nest_desc* desc, int64_t nro
     if ((s = prepare_fallback(p, &fb, stream)) != NEST_OK) return s;
     cudaStream_t st = as_stream(stream);
     cudaError_t e;
+    const int nchunks = staged || p.x_halo > 0 ? 1 : hostio_chunks(nnz);
+    if (nchunks > 1)
+        return spmv_hostio_pipelined(desc, nchunks, nrows, ncols, nnz, h_rowptr, h_colind, h_val, h_x, h_y,
+                                     d_rowptr, d_col, d_val, d_x, d_y, fb, st);
     if ((e = cudaMemcpyAsync(d_rowptr, h_rowptr, (size_t)(nrows + 1) * 8, cudaMemcpyHostToDevice, st)) ||
         (nnz && (e = cudaMemcpyAsync(d_col, h_colind, (size_t)nnz * 4, cudaMemcpyHostToDevice, st))) ||
         (nnz && (e = cudaMemcpyAsync(d_val, h_val, (size_t)nnz * 8, cudaMemcpyHostToDevice, st))) ||
@@ -542,5 +683,11 @@ NEST_API nest_status nest_shutdown(void) {
         }
     }
     if (first != cudaSuccess) return cuda_fail(first, "cudaFree(fallback)");
+    std::lock_guard<std::mutex> lk2(g_hostio_mu);
+    auto h = g_hostio.find(dev);
+    if (h != g_hostio.end()) {
+        hostio_destroy(h->second);
+        g_hostio.erase(h);
+    }
     return NEST_OK;
 }
