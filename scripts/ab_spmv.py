@@ -21,6 +21,9 @@ CFGS = {
     "S2 bv": dict(simdlen=2, threads_per_team=1024, blocked=True, vec128=True),
     "S1 bv": dict(simdlen=1, threads_per_team=1024, blocked=True, vec128=True),
     "S2 b": dict(simdlen=2, threads_per_team=1024, blocked=True),
+    "S2 bvh": dict(simdlen=2, threads_per_team=1024, blocked=True, vec128=True, stream_hints=True),
+    "S1 bvh": dict(simdlen=1, threads_per_team=1024, blocked=True, vec128=True, stream_hints=True),
+    "S4 bvh": dict(simdlen=4, threads_per_team=1024, blocked=True, vec128=True, stream_hints=True),
     "S1 cyc256": dict(simdlen=1, threads_per_team=256),
     "S2 bv T768": dict(simdlen=2, threads_per_team=768, blocked=True, vec128=True),
     "S1 bv T768": dict(simdlen=1, threads_per_team=768, blocked=True, vec128=True),
