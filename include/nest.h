@@ -109,7 +109,8 @@ enum {
      * grid.  Results are identical (the schedule never changes a row's
      * arithmetic). */
     NEST_F_BLOCKED = 1u << 3,
-    /* 128-bit loads (SpMV; batched matvec: float4 tuples of a row, needs
+    /* 128-bit loads (SpMV; nested stencil: pairs of inner iterations, see
+     * nest_nested_stencil_f64; batched matvec: float4 tuples of a row, needs
      * n % 4 == 0 and 16-byte aligned A and x).  SpMV: the simd loop runs over pairs of nonzeros
      * (one 128-bit val load, one 64-bit colind load per pair), lane l taking
      * pairs l, l+S, ... of the row ("blocked-cyclic" order: real results
@@ -211,7 +212,11 @@ nest_status nest_batched_matvec_f32(const nest_desc *desc, int64_t batch, int32_
  *   s = (+)_{j<trip} coef[j] * ((in[base+j-1] + 2*in[base+j]) + in[base+j+1]);
  *   out[i] = trip == 0 ? +0.0 : scale * s.
  * in f64[nouter*L+2], coef f64[L], w f64[nouter], out f64[nouter];
- * visits: one u64 accumulated into (may be NULL). */
+ * visits: one u64 accumulated into (may be NULL).  NEST_F_VEC128: the simd
+ * unit is a pair of inner iterations (two 128-bit loads of in, one of coef per
+ * pair); needs an even L and 16-byte aligned in and coef (else
+ * NEST_ERR_UNSUPPORTED); real results differ from the scalar lane order by
+ * rounding only. */
 nest_status nest_nested_stencil_f64(const nest_desc *desc, int64_t nouter, int32_t L,
                                     const double *in, const double *coef, const double *w,
                                     double *out, unsigned long long *visits, void *stream);

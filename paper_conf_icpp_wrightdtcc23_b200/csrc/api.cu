@@ -609,6 +609,9 @@ NEST_API nest_status nest_nested_stencil_f64(const nest_desc* desc, int64_t nout
     if (s != NEST_OK) return s;
     if (nouter == 0) return NEST_OK;
     if (!w || !out || (L > 0 && (!in || !coef))) return fail(NEST_ERR_INVALID_ARG, "in/coef/w/out is NULL");
+    if ((p.flags & NEST_F_VEC128) &&
+        ((L & 1) || (reinterpret_cast<uintptr_t>(in) & 15) || (reinterpret_cast<uintptr_t>(coef) & 15)))
+        return fail(NEST_ERR_UNSUPPORTED, "NEST_F_VEC128 (stencil) needs an even L and 16-byte aligned in and coef");
     unsigned char* fb = nullptr;
     if ((s = prepare_fallback(p, &fb, stream)) != NEST_OK) return s;
     return launch_stencil(p, nouter, L, in, coef, w, out, visits, fb, as_stream(stream));

@@ -558,6 +558,36 @@ struct StencilBody {
     }
 };
 
+// a10 with 128-bit tuples (NEST_F_VEC128, even L, 16-byte aligned in/coef):
+// simd unit = a pair of consecutive inner iterations (j = 2t, 2t+1).  The
+// pair's four neighbours in[p-1 .. p+2] are two aligned double2 loads (p - 1 =
+// i*L + 2t is even) and its coefficients one, against eight scalar loads for
+// two elements in StencilBody; each element's t and fma are StencilBody's, in
+// the same j order within the lane (the lanes' partial sums cover different j
+// sets, so real-valued results match the oracle to the R3 tolerance and
+// integer-valued ones bit for bit).  Measured motivation: the SPMD stencil is
+// issue-bound at S >= 8 (profiles/r01s3_mode_study.md).
+struct StencilVecBody : StencilBody {
+    __device__ __forceinline__ Loop prologue(int64_t i, int k, Step& st, bool side_effects,
+                                             TeamShared& tsh) const {
+        Loop l = StencilBody::prologue(i, k, st, side_effects, tsh);
+        l.trip >>= 1;   // L / 2 pairs
+        return l;
+    }
+    template <int OP>
+    __device__ __forceinline__ double accum(const Loop& Lp, int64_t t, double acc) const {
+        const int64_t j = 2 * t;
+        const double* p = in + Lp.base + j;
+        const double2 a = __ldg(reinterpret_cast<const double2*>(p - 1));   // in[p-1], in[p]
+        const double2 b = __ldg(reinterpret_cast<const double2*>(p + 1));   // in[p+1], in[p+2]
+        const double2 c = __ldg(reinterpret_cast<const double2*>(coef + j));
+        const double t0 = (a.x + 2.0 * a.y) + b.x;
+        const double t1 = (a.y + 2.0 * b.x) + b.y;
+        acc = Red<OP, double>::accum(acc, c.x, t0);
+        return Red<OP, double>::accum(acc, c.y, t1);
+    }
+};
+
 // ------------------------------------------------ NEXT-2 laplace3d
 // 3-D heat-diffusion step (the Fig 10 cost study):
 // teams distribute + parallel for over the (i, j) lines of the interior, simd

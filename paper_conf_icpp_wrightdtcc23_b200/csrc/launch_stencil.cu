@@ -15,7 +15,9 @@ int32_t stencil_payload(int32_t U) {
 nest_status launch_stencil(const Plan& p, int64_t, int32_t L, const double* in, const double* coef,
                            const double* w, double* out, unsigned long long* visits,
                            unsigned char* fb, cudaStream_t st) {
-    return dispatch(p, StencilBody{in, coef, w, out, visits, L}, fb, st);
+    const StencilBody b{in, coef, w, out, visits, L};
+    if (p.flags & NEST_F_VEC128) return dispatch(p, StencilVecBody{b}, fb, st);
+    return dispatch(p, b, fb, st);
 }
 
 }  // namespace nest

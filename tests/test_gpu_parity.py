@@ -578,3 +578,42 @@ def test_spmv_teams_generic_baseline(P, cfg1, banded):
     yr2, _ = oracle.spmv_csr_f64(rp2, col2, val2, x2)
     y2 = host(P.spmv_csr_f64(dev(rp2), dev(col2), dev(val2), dev(x2), simdlen=1, mode="teams_generic"))
     assert np.array_equal(bits(y2), bits(yr2))
+
+
+# ------------------------------------------------------------------ a10 stencil, 128-bit pairs
+@pytest.mark.parametrize("L", (2, 4, 8, 16, 32, 64, 34))
+@pytest.mark.parametrize("mode", MODES)
+def test_stencil_vec128(P, L, mode):
+    """Pair tuples (NEST_F_VEC128): integer data bit-exact against the oracle,
+    real data within R3; every simdlen, U = 1/2; the guarded visit count once per i."""
+    N = 4099
+    for values in ("int", "real"):
+        inp, coef, w = R.stencil_inputs(N, L, values=values)
+        yref, aref, vref = oracle.nested_stencil_f64(inp, coef, w, N, L)
+        t = [dev(inp), dev(coef), dev(w)]
+        for S in SIMDLENS:
+            for U in (1, 2):
+                visits = torch.zeros(1, dtype=torch.int64, device="cuda")
+                y = host(P.nested_stencil_f64(*t, N, L, visits=visits, simdlen=S, mode=mode, outer_unroll=U,
+                                              vec128=True))
+                assert int(visits.item()) == vref == N
+                if values == "int":
+                    assert np.array_equal(bits(y), bits(yref)), (S, U)
+                else:
+                    assert_close(y, yref, aref, 1e-12)
+
+
+def test_stencil_vec128_full_and_rejects(P):
+    N = 1 << 20
+    for L in (4, 64):
+        inp, coef, w = R.stencil_inputs(N, L)
+        yref, aref, _ = oracle.nested_stencil_f64(inp, coef, w, N, L)
+        t = [dev(inp), dev(coef), dev(w)]
+        for S in (2, 8, 32):
+            y = host(P.nested_stencil_f64(*t, N, L, simdlen=S, vec128=True))
+            assert_close(y, yref, aref, 1e-12)
+        ymax, _, _ = oracle.nested_stencil_f64(inp, coef, w, N, L, op="max")
+        assert np.array_equal(host(P.nested_stencil_f64(*t, N, L, simdlen=16, reduce="max", vec128=True)), ymax)
+    inp, coef, w = R.stencil_inputs(64, 3)
+    with pytest.raises(Exception, match="even L"):
+        P.nested_stencil_f64(dev(inp), dev(coef), dev(w), 64, 3, vec128=True)
