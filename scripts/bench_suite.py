@@ -83,21 +83,29 @@ def cfg3(out):
                 if S == 1 and mode != "spmd":
                     continue
                 for blocked in (False, True):
-                    ms = timed_graph(lambda: P.nested_stencil_f64(*t, N, L, o, simdlen=S, mode=mode,
-                                                                  blocked=blocked, threads_per_team=256))
-                    res.append(dict(L=L, S=S, mode=mode, blocked=blocked, ms=ms, GBs=B / ms / 1e6))
+                    for vec in (False, True):   # scalar simd unit / 128-bit pairs (StencilVecBody)
+                        ms = timed_graph(lambda: P.nested_stencil_f64(*t, N, L, o, simdlen=S, mode=mode,
+                                                                      blocked=blocked, threads_per_team=256,
+                                                                      vec128=vec))
+                        res.append(dict(L=L, S=S, mode=mode, blocked=blocked, vec=vec, ms=ms, GBs=B / ms / 1e6))
         print("cfg3 L", L, "done", flush=True)
     summary = {}
     for L in R.STENCIL_LS:
-        rows = [r for r in res if r["L"] == L]
-        best = min(rows, key=lambda r: r["ms"])
-        s1 = min((r for r in rows if r["S"] == 1), key=lambda r: r["ms"])
+        allrows = [r for r in res if r["L"] == L]
+        best = min(allrows, key=lambda r: r["ms"])
+        s1 = min((r for r in allrows if r["S"] == 1), key=lambda r: r["ms"])
+        # the mode study (generic / SPMD at each simdlen) on the scalar simd unit
+        rows = [r for r in allrows if not r["vec"]]
+        best_scalar = min(rows, key=lambda r: r["ms"])
+        s1_scalar = min((r for r in rows if r["S"] == 1), key=lambda r: r["ms"])
         ratios = {}
         for S in (2, 4, 8, 16, 32):
             sp = min((r["ms"] for r in rows if r["S"] == S and r["mode"] == "spmd"))
             ratios[S] = {m: min(r["ms"] for r in rows if r["S"] == S and r["mode"] == m) / sp
                          for m in ("generic_smem", "generic_shfl")}
         summary[L] = dict(best=best, simdlen1=s1, speedup_vs_simdlen1=s1["ms"] / best["ms"],
+                          best_scalar=best_scalar,
+                          scalar_speedup_vs_simdlen1=s1_scalar["ms"] / best_scalar["ms"],
                           generic_over_spmd=ratios)
     out["cfg3"] = dict(note="N=2^20 outer iterations; 20 launches captured in a CUDA graph, replayed per event pair "
                             "(no flush, no host launch overhead)",
