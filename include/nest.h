@@ -228,7 +228,10 @@ nest_status nest_nested_stencil_f64(const nest_desc *desc, int64_t nouter, int32
  *            + u[i][j][k-1]) + u[i][j][k+1]) - 6*u[i][j][k]
  *   out[i][j][k] = u[i][j][k] + alpha*lap      (no FMA contraction)
  * Boundary points of out are not written.  Outer (parallel) unit = a line
- * (i, j), simd unit = k.  u and out must not alias. */
+ * (i, j), simd unit = k.  u and out must not alias.  NEST_F_VEC128: the simd
+ * unit is the aligned pair k = 2t, 2t+1 (t < nx/2; boundary points computed
+ * but not stored); needs an even nx and 16-byte aligned u and out (else
+ * NEST_ERR_UNSUPPORTED); results are bit-identical to the scalar unit. */
 nest_status nest_laplace3d_f64(const nest_desc *desc, int64_t nz, int64_t ny, int64_t nx,
                                double alpha, const double *u, double *out, void *stream);
 

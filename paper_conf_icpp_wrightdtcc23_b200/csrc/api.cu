@@ -627,6 +627,9 @@ NEST_API nest_status nest_laplace3d_f64(const nest_desc* desc, int64_t nz, int64
     if (lines == 0 || nx <= 2) return NEST_OK;
     if (!u || !out) return fail(NEST_ERR_INVALID_ARG, "u/out is NULL");
     if (u == out) return fail(NEST_ERR_INVALID_ARG, "u and out must not alias (Jacobi step)");
+    if ((p.flags & NEST_F_VEC128) &&
+        ((nx & 1) || (reinterpret_cast<uintptr_t>(u) & 15) || (reinterpret_cast<uintptr_t>(out) & 15)))
+        return fail(NEST_ERR_UNSUPPORTED, "NEST_F_VEC128 (laplace3d) needs an even nx and 16-byte aligned u and out");
     unsigned char* fb = nullptr;
     if ((s = prepare_fallback(p, &fb, stream)) != NEST_OK) return s;
     return launch_laplace(p, nz, ny, nx, alpha, u, out, fb, as_stream(stream));

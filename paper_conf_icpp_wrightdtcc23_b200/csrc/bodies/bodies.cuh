@@ -650,6 +650,49 @@ struct LaplaceBody {
     __device__ __forceinline__ void epilogue(const Step&, double) const {}
 };
 
+// NEXT-2 with 128-bit pairs (NEST_F_VEC128, even nx, 16-byte aligned u/out):
+// the simd unit is the aligned pair k = 2t, 2t+1 of a line (t < nx/2), so every
+// neighbour pair (z-1, z+1, y-1, y+1, the centres) is one double2 load and only
+// u[k-1], u[k+2] are scalar: 7 loads per two points against 14.  Each point's
+// arithmetic is LaplaceBody's, operand for operand (bit-identical to the
+// oracle); the line's boundary points k = 0 and nx-1 are computed from valid
+// neighbouring memory (interior lines only) and not stored.
+struct LaplaceVecBody : LaplaceBody {
+    __device__ __forceinline__ Loop prologue(int64_t o, int k, Step& st, bool se, TeamShared& t) const {
+        Loop l = LaplaceBody::prologue(o, k, st, se, t);
+        return Loop{nx >> 1, l.base - 1};   // pairs over the whole line, base = line start
+    }
+    static __device__ __forceinline__ double point(double zm, double zp, double ym, double yp, double xm,
+                                                   double xp, double uc, double alpha) {
+        double lap = __dadd_rn(zm, zp);
+        lap = __dadd_rn(lap, ym);
+        lap = __dadd_rn(lap, yp);
+        lap = __dadd_rn(lap, xm);
+        lap = __dadd_rn(lap, xp);
+        lap = __dsub_rn(lap, __dmul_rn(6.0, uc));
+        return __dadd_rn(uc, __dmul_rn(alpha, lap));
+    }
+    __device__ __forceinline__ void apply(const Loop& L, int64_t t) const {
+        const int64_t k0 = 2 * t;
+        const int64_t c = L.base + k0;
+        const int64_t sz = ny * nx;
+        const double2 zm = __ldg(reinterpret_cast<const double2*>(u + c - sz));
+        const double2 zp = __ldg(reinterpret_cast<const double2*>(u + c + sz));
+        const double2 ym = __ldg(reinterpret_cast<const double2*>(u + c - nx));
+        const double2 yp = __ldg(reinterpret_cast<const double2*>(u + c + nx));
+        const double2 uc = __ldg(reinterpret_cast<const double2*>(u + c));
+        const double xm = __ldg(u + c - 1), xp = __ldg(u + c + 2);
+        const double o0 = point(zm.x, zp.x, ym.x, yp.x, xm, uc.y, uc.x, alpha);
+        const double o1 = point(zm.y, zp.y, ym.y, yp.y, uc.x, xp, uc.y, alpha);
+        if (k0 >= 1 && k0 + 1 <= nx - 2) {
+            *reinterpret_cast<double2*>(out + c) = make_double2(o0, o1);
+        } else {
+            if (k0 >= 1 && k0 <= nx - 2) out[c] = o0;
+            if (k0 + 1 >= 1 && k0 + 1 <= nx - 2) out[c + 1] = o1;
+        }
+    }
+};
+
 // ---------------------------------------------------------------- probe
 // One outer iteration per group; the simd loop body records coverage (hits),
 // the executing lane (owner, group 0 only) and counts iterations through the

@@ -15,7 +15,9 @@ int32_t laplace_payload(int32_t U) {
 nest_status launch_laplace(const Plan& p, int64_t nz, int64_t ny, int64_t nx, double alpha, const double* u,
                            double* out, unsigned char* fb, cudaStream_t st) {
     (void)nz;
-    return dispatch(p, LaplaceBody{u, out, ny, nx, alpha}, fb, st);
+    const LaplaceBody b{u, out, ny, nx, alpha};
+    if (p.flags & NEST_F_VEC128) return dispatch(p, LaplaceVecBody{b}, fb, st);
+    return dispatch(p, b, fb, st);
 }
 
 }  // namespace nest

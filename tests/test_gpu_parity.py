@@ -617,3 +617,25 @@ def test_stencil_vec128_full_and_rejects(P):
     inp, coef, w = R.stencil_inputs(64, 3)
     with pytest.raises(Exception, match="even L"):
         P.nested_stencil_f64(dev(inp), dev(coef), dev(w), 64, 3, vec128=True)
+
+
+@pytest.mark.parametrize("S", SIMDLENS)
+@pytest.mark.parametrize("mode", MODES)
+def test_laplace3d_vec128(P, S, mode):
+    """Aligned pairs over whole lines (NEST_F_VEC128, even nx): bit-identical to the
+    oracle, boundary points untouched."""
+    for (nz, ny, nx), values in (((9, 11, 38), "real"), ((5, 34, 66), "int"), ((3, 3, 4), "real"),
+                                 ((4, 5, 2), "real"), ((6, 7, 130), "real")):
+        u = R.laplace_inputs(nz, ny, nx, values=values)
+        ref = oracle.laplace3d_f64(u, nz, ny, nx, 0.125)
+        for U, blocked in ((1, False), (2, True), (4, False)):
+            out = dev(u.copy())
+            P.laplace3d_f64(dev(u), out, nz, ny, nx, 0.125, simdlen=S, mode=mode, outer_unroll=U, blocked=blocked,
+                            vec128=True)
+            assert np.array_equal(bits(host(out)), bits(ref)), (nz, ny, nx, U, blocked)
+
+
+def test_laplace3d_vec128_rejects_odd_nx(P):
+    u = R.laplace_inputs(4, 4, 5)
+    with pytest.raises(Exception, match="even nx"):
+        P.laplace3d_f64(dev(u), dev(u.copy()), 4, 4, 5, 0.125, vec128=True)
