@@ -657,7 +657,11 @@ struct LaplaceBody {
 // arithmetic is LaplaceBody's, operand for operand (bit-identical to the
 // oracle); the line's boundary points k = 0 and nx-1 are computed from valid
 // neighbouring memory (interior lines only) and not stored.
+#ifndef NEST_LAPLACE_2PM
+#define NEST_LAPLACE_2PM 0   // A/B switch: 2 teams of 1024 per SM (32-register cap) at U = 1
+#endif
 struct LaplaceVecBody : LaplaceBody {
+    static constexpr bool two_teams_for(int) { return NEST_LAPLACE_2PM != 0; }
     __device__ __forceinline__ Loop prologue(int64_t o, int k, Step& st, bool se, TeamShared& t) const {
         Loop l = LaplaceBody::prologue(o, k, st, se, t);
         return Loop{nx >> 1, l.base - 1};   // pairs over the whole line, base = line start

@@ -11,7 +11,7 @@ FL="-O3 -std=c++17 -gencode arch=compute_100a,code=sm_100a -lineinfo -Xcompiler 
 mkdir -p build_$name
 for f in paper_conf_icpp_wrightdtcc23_b200/csrc/*.cu; do
   b=$(basename $f .cu)
-  if [ -n "$VARIANT_ALL" ] || grep -q "SpmvVecBody\|BatchedVecBody\|StencilBody" $f || [ $b = spmv_vec2 ] || [ $b = spmv_vec4 ]; then
+  if [ -n "$VARIANT_ALL" ] || grep -q "SpmvVecBody\|BatchedVecBody\|StencilBody\|LaplaceVecBody" $f || [ $b = spmv_vec2 ] || [ $b = spmv_vec4 ]; then
     nvcc $FL "$@" -c $f -o build_$name/$b.o &
   else
     cp build/$b.o build_$name/$b.o
