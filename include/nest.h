@@ -93,14 +93,7 @@ enum {
      * with L1 no-allocate / L2 evict-first loads; 128-bit path -- the CSR
      * tuples with L1 no-allocate loads (L1 kept for the x gathers). */
     NEST_F_STREAM_HINTS = 1u << 1,
-    /* SpMV only: warp-specialised pipeline.  Warp 0 of each team stages the
-     * team's row chunks (rowptr, colind, val and, with x_halo > 0, the x
-     * window) into shared memory with bulk asynchronous copies (TMA engine) and
-     * mbarriers; warps 1-2 gather x for the staged nonzeros (window hits from
-     * shared memory, the rest with asynchronous copies); warps 3.. run the loop
-     * nest out of shared memory.  Needs threads_per_team >= 128 and 16-byte
-     * aligned colind, val and x.  Results are identical to the unstaged path. */
-    NEST_F_STAGED = 1u << 2,
+    /* bit 2 is reserved (an earlier staged-pipeline variant; rejected as an unknown flag). */
     /* "teams distribute" with a static block schedule: team b owns the
      * contiguous outer range [b*C, (b+1)*C) (C = ceil(outer / grid) rounded up
      * to a multiple of G, or team_chunk: then chunks b, b + grid, ...) and its
@@ -134,27 +127,51 @@ typedef struct {
     int32_t sharing_bytes;      /* generic sharing space per team; 0 = 2048 */
     uint32_t flags;             /* NEST_F_* */
     int32_t outer_unroll;       /* U: outer iterations a group keeps in flight (1, 2, 4); 0 = 1 */
-    int32_t x_halo;             /* SpMV only. > 0: stage x in shared memory as a sliding window
-                                 * [row0 - x_halo, row0 + rows + x_halo) around each team's chunk of
-                                 * rows (banded matrices); columns outside it read global memory.
-                                 * Results are identical; 0 = no staging. */
+    int32_t x_halo;             /* SpMV only.  H > 0: the x ring.  Each team owns a
+                                 * contiguous range of rows and walks it in rounds of R = G*U rows
+                                 * (G = (T - 32)/S consumer groups; here outer_unroll U is the rows a
+                                 * group runs per round, one after another); its last warp bulk-copies
+                                 * (TMA engine) each round's row bounds and the x window
+                                 * [row0 - H, row0 + R + H) into shared-memory rings ahead of use, with
+                                 * mbarriers instead of team barriers.  Columns inside the window read
+                                 * the ring, others read x in global memory: results are identical for
+                                 * every H (bit-identical to nest_kernel at the same S, mode and loads).
+                                 * Needs T >= 64 and 16-byte aligned x; scalar or pair loads (not
+                                 * quads); pairs need nnz, nrows < 2^31.  0 = no ring. */
     int32_t team_chunk;         /* with NEST_F_BLOCKED: outer iterations per team chunk, rounded up to
                                  * a multiple of G; team b takes chunks b, b + grid, b + 2 grid, ...
                                  * (its groups cyclically inside a chunk), so all teams sweep the
                                  * outer range together.  0 = one contiguous range per team. */
-    int32_t reserved;           /* must be 0 */
+    int32_t teams_per_sm;       /* x ring only: teams sharing an SM that the rings are sized for
+                                 * (1 or 2; 0 = the planner's choice).  Two teams of
+                                 * 1024 get 32 registers per thread and ~94 KB of ring each; one team
+                                 * gets 64 registers and ~190 KB.  Must be 0 without x_halo. */
 } nest_desc;
+
+/* Which kernel an SpMV plan launches (nest_plan_info.kernel). */
+enum {
+    NEST_KERNEL_NEST = 0,           /* nest_kernel: the loop-nest engine (engine.cuh) */
+    NEST_KERNEL_XRING = 1,          /* spmv_ring_kernel: x_halo > 0 (device/spmv_ring.cuh) */
+    NEST_KERNEL_TEAMS_GENERIC = 2   /* NEXT-1 two-level baseline (device/teams_generic.cuh) */
+};
 
 /* Resolved launch geometry (a1). */
 typedef struct {
     int32_t grid;                 /* teams (blocks) */
     int32_t block;                /* threads per team T */
-    int32_t groups_per_team;      /* G = T / S */
-    int32_t slot_bytes;           /* sharing_bytes / G (generic-SMEM slot per group) */
-    int32_t payload_bytes;        /* bytes one group posts per simd batch */
-    int32_t uses_global_fallback; /* payload_bytes > slot_bytes (GENERIC_SMEM only) */
+    int32_t groups_per_team;      /* G = T / S (x ring: (T - 32) / S consumer groups) */
+    int32_t slot_bytes;           /* sharing_bytes / G rounded down to 8 (generic-SMEM slot per group) */
+    int32_t payload_bytes;        /* bytes one group posts per simd batch (nest_spmv_plan: of the body
+                                   * that actually runs) */
+    int32_t uses_global_fallback; /* payload_bytes > slot_bytes (GENERIC_SMEM only); the kernel
+                                   * follows this decision */
     int32_t outer_unroll;         /* U */
     int32_t smem_bytes;           /* dynamic shared memory per team */
+    int32_t kernel;               /* NEST_KERNEL_* */
+    int32_t index_bits;           /* 32 or 64: row / nonzero index width of the launched body */
+    int32_t ring_segments;        /* x ring: segment slots of 256 doubles (else 0) */
+    int32_t ring_row_slots;       /* x ring: row-bound slots (else 0) */
+    int64_t chunk;                /* blocked schedule / x ring: outer iterations per team chunk (else 0) */
 } nest_plan_info;
 
 uint32_t nest_abi_version(void);
@@ -168,6 +185,15 @@ const char *nest_last_error(void);
  * device (NEST_ERR_CUDA without one).  Errors: NEST_ERR_INVALID_ARG. */
 nest_status nest_plan(const nest_desc *desc, int64_t outer_iters, int32_t payload_bytes,
                       nest_plan_info *out);
+
+/* a1 for a8: the plan nest_spmv_csr_f64 launches for this descriptor and
+ * matrix shape -- kernel, geometry, index width, x-ring sizing, and the payload
+ * of the body that runs, so uses_global_fallback is exactly the kernel's
+ * choice.  Queries the current device when the grid is sized from occupancy
+ * (num_teams == 0 with a persistent/blocked grid, a fallback, or the x ring).
+ * Errors: as nest_spmv_csr_f64's validation. */
+nest_status nest_spmv_plan(const nest_desc *desc, int64_t nrows, int64_t ncols, int64_t nnz,
+                           nest_plan_info *out);
 
 /* a8: CSR SpMV, y[i] = (+)_{k in [rowptr[i], rowptr[i+1])} val[k] * x[colind[k]]
  * (sparse_matvec).  Outer (parallel) unit = a row; simd
@@ -189,8 +215,11 @@ nest_status nest_spmv_csr_f64(const nest_desc *desc, int64_t nrows, int64_t ncol
  * on it before the call, and work queued on it after the call starts after
  * the last y row is on the host.  Results equal nest_spmv_csr_f64's bit for
  * bit.  rowptr must start at 0 and end at nnz.  The host buffers must stay
- * valid, and h_y unread, until `stream` reaches that point.  Staged and
- * x_halo variants copy in one shot. */
+ * valid, and h_y unread, until `stream` reaches that point.  d_workspace must
+ * be 256-byte aligned.  The H2D/D2H streams and events are library-owned, one
+ * set per device, guarded by a lock: concurrent callers on one device
+ * serialise their enqueueing (not their kernels).  Pageable host buffers work
+ * but make the copies synchronous. */
 size_t nest_spmv_hostio_workspace_bytes(int64_t nrows, int64_t ncols, int64_t nnz);
 nest_status nest_spmv_csr_f64_hostio(const nest_desc *desc, int64_t nrows, int64_t ncols,
                                      int64_t nnz, const int64_t *h_rowptr,
@@ -355,8 +384,8 @@ nest_status nest_xpeer_barrier(nest_xpeer *xp, void *stream);
  * caller may overwrite its slice on return).  Arguments as
  * nest_spmv_csr_f64_dist (GLOBAL column indices, 0-based local rowptr).
  * Variants: the cyclic / blocked schedules, scalar or 128-bit pair loads
- * (NEST_F_VEC128 without NEST_F_VEC_QUAD); NEST_F_STAGED, x_halo and
- * NEST_MODE_TEAMS_GENERIC return NEST_ERR_UNSUPPORTED. */
+ * (NEST_F_VEC128 without NEST_F_VEC_QUAD); x_halo and NEST_MODE_TEAMS_GENERIC
+ * return NEST_ERR_UNSUPPORTED. */
 nest_status nest_spmv_csr_f64_xpeer(const nest_desc *desc, nest_xpeer *xp, int64_t nrows_global,
                                     int64_t nrows_local, int64_t nnz_local, const int64_t *rowptr_local,
                                     const int32_t *colind, const double *val, double *y_local,

@@ -24,10 +24,10 @@ NEST_MODE_SPMD, NEST_MODE_GENERIC_SMEM, NEST_MODE_GENERIC_SHFL, NEST_MODE_TEAMS_
 NEST_REDUCE_SUM, NEST_REDUCE_MAX, NEST_REDUCE_MIN = 0, 1, 2
 NEST_F_PERSISTENT_GRID = 1 << 0
 NEST_F_STREAM_HINTS = 1 << 1
-NEST_F_STAGED = 1 << 2
 NEST_F_BLOCKED = 1 << 3
 NEST_F_VEC128 = 1 << 4
 NEST_F_VEC_QUAD = 1 << 5
+NEST_KERNEL_NEST, NEST_KERNEL_XRING, NEST_KERNEL_TEAMS_GENERIC = 0, 1, 2
 
 
 class nest_desc(ctypes.Structure):
@@ -36,7 +36,7 @@ class nest_desc(ctypes.Structure):
                 ("mode", ctypes.c_int32), ("reduce", ctypes.c_int32),
                 ("sharing_bytes", ctypes.c_int32), ("flags", ctypes.c_uint32),
                 ("outer_unroll", ctypes.c_int32), ("x_halo", ctypes.c_int32),
-                ("team_chunk", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+                ("team_chunk", ctypes.c_int32), ("teams_per_sm", ctypes.c_int32)]
 
 
 NEST_MAX_REGIONS = 4
@@ -53,7 +53,10 @@ class nest_plan_info(ctypes.Structure):
     _fields_ = [("grid", ctypes.c_int32), ("block", ctypes.c_int32),
                 ("groups_per_team", ctypes.c_int32), ("slot_bytes", ctypes.c_int32),
                 ("payload_bytes", ctypes.c_int32), ("uses_global_fallback", ctypes.c_int32),
-                ("outer_unroll", ctypes.c_int32), ("smem_bytes", ctypes.c_int32)]
+                ("outer_unroll", ctypes.c_int32), ("smem_bytes", ctypes.c_int32),
+                ("kernel", ctypes.c_int32), ("index_bits", ctypes.c_int32),
+                ("ring_segments", ctypes.c_int32), ("ring_row_slots", ctypes.c_int32),
+                ("chunk", ctypes.c_int64)]
 
 
 _i32, _i64, _u32, _vp, _sz = ctypes.c_int32, ctypes.c_int64, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_size_t
@@ -66,6 +69,7 @@ SIGNATURES = {
     "nest_status_str": (ctypes.c_char_p, [_st]),
     "nest_last_error": (ctypes.c_char_p, []),
     "nest_plan": (_st, [_D, _i64, _i32, ctypes.POINTER(nest_plan_info)]),
+    "nest_spmv_plan": (_st, [_D, _i64, _i64, _i64, ctypes.POINTER(nest_plan_info)]),
     "nest_spmv_csr_f64": (_st, [_D, _i64, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp]),
     "nest_spmv_hostio_workspace_bytes": (_sz, [_i64, _i64, _i64]),
     "nest_spmv_csr_f64_hostio": (_st, [_D, _i64, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _sz, _vp]),

@@ -32,8 +32,8 @@ def check(status: int, where: str) -> None:
 def make_desc(simdlen: int = 8, mode: str | int = "spmd", reduce: str | int = "sum",
               threads_per_team: int = 256, num_teams: int = 0, sharing_bytes: int = 0,
               outer_unroll: int = 1, persistent: bool = False, stream_hints: bool = False,
-              x_halo: int = 0, staged: bool = False, blocked: bool = False,
-              vec128: bool = False, quad: bool = False, team_chunk: int = 0,
+              x_halo: int = 0, blocked: bool = False,
+              vec128: bool = False, quad: bool = False, team_chunk: int = 0, teams_per_sm: int = 0,
               flags: int = 0) -> N.nest_desc:
     d = N.nest_desc()
     d.abi_version = N.NEST_ABI_VERSION
@@ -46,8 +46,9 @@ def make_desc(simdlen: int = 8, mode: str | int = "spmd", reduce: str | int = "s
     d.outer_unroll = outer_unroll
     d.x_halo = x_halo
     d.team_chunk = team_chunk
+    d.teams_per_sm = teams_per_sm
     d.flags = flags | (N.NEST_F_PERSISTENT_GRID if persistent else 0) | (
-        N.NEST_F_STREAM_HINTS if stream_hints else 0) | (N.NEST_F_STAGED if staged else 0) | (
+        N.NEST_F_STREAM_HINTS if stream_hints else 0) | (
         N.NEST_F_BLOCKED if blocked else 0) | (N.NEST_F_VEC128 if vec128 or quad else 0) | (
         N.NEST_F_VEC_QUAD if quad else 0)
     return d
@@ -57,6 +58,14 @@ def plan(outer_iters: int, payload_bytes: int = 0, **cfg) -> dict:
     info = N.nest_plan_info()
     check(N.nest_plan(ctypes.byref(make_desc(**cfg)), outer_iters, payload_bytes,
                       ctypes.byref(info)), "nest_plan")
+    return {f: getattr(info, f) for f, _ in N.nest_plan_info._fields_}
+
+
+def spmv_plan(nrows: int, ncols: int, nnz: int, **cfg) -> dict:
+    """a1 for a8: the plan nest_spmv_csr_f64 launches for this matrix shape."""
+    info = N.nest_plan_info()
+    check(N.nest_spmv_plan(ctypes.byref(make_desc(**cfg)), nrows, ncols, nnz, ctypes.byref(info)),
+          "nest_spmv_plan")
     return {f: getattr(info, f) for f, _ in N.nest_plan_info._fields_}
 
 
@@ -112,11 +121,13 @@ def spmv_csr_f64_hostio(h_rowptr, h_colind, h_val, h_x, h_y, workspace, *, strea
     torch = _torch()
     nrows = h_rowptr.numel() - 1
     ncols, nnz = h_x.numel(), h_val.numel()
-    for t, dt, name in ((h_rowptr, torch.int64, "h_rowptr"), (h_colind, torch.int32, "h_colind"),
-                        (h_val, torch.float64, "h_val"), (h_x, torch.float64, "h_x"),
-                        (h_y, torch.float64, "h_y")):
+    for t, dt, name, n in ((h_rowptr, torch.int64, "h_rowptr", nrows + 1), (h_colind, torch.int32, "h_colind", nnz),
+                           (h_val, torch.float64, "h_val", nnz), (h_x, torch.float64, "h_x", ncols),
+                           (h_y, torch.float64, "h_y", nrows)):
         if t.is_cuda or t.dtype != dt or not t.is_contiguous():
             raise TypeError(f"{name} must be a contiguous host {dt} tensor")
+        if t.numel() < n:   # the C side copies n elements from / into it
+            raise ValueError(f"{name} has {t.numel()} elements, needs {n}")
     d = make_desc(**cfg)
     check(N.nest_spmv_csr_f64_hostio(ctypes.byref(d), nrows, ncols, nnz,
                                      ctypes.c_void_p(h_rowptr.data_ptr()),

@@ -51,7 +51,6 @@ static constexpr int32_t kMaxBlocksPerSm = 32;
 static constexpr int32_t kMaxThreadsPerSm = 2048;
 static constexpr int32_t kSmemPerSm = 228 * 1024;
 static constexpr int32_t kSmemReservedPerBlock = 1024;
-static constexpr int32_t kMaxDynSmem = 227 * 1024;
 
 // Descriptor validation (groups are equal,
 // inside one warp, and divide the team evenly).
@@ -79,10 +78,13 @@ static nest_status validate_desc(const nest_desc* d, int32_t* T, int32_t* sharin
     *U = d->outer_unroll ? d->outer_unroll : 1;
     if (*U != 1 && *U != 2 && *U != 4)
         return fail(NEST_ERR_INVALID_ARG, "outer_unroll %d: need 1, 2 or 4", d->outer_unroll);
-    if (d->flags & ~(uint32_t)(NEST_F_PERSISTENT_GRID | NEST_F_STREAM_HINTS | NEST_F_STAGED | NEST_F_BLOCKED |
+    if (d->flags & ~(uint32_t)(NEST_F_PERSISTENT_GRID | NEST_F_STREAM_HINTS | NEST_F_BLOCKED |
                                NEST_F_VEC128 | NEST_F_VEC_QUAD))
         return fail(NEST_ERR_INVALID_ARG, "unknown flags 0x%x", d->flags);
-    if (d->reserved) return fail(NEST_ERR_INVALID_ARG, "reserved fields must be 0");
+    if (d->teams_per_sm < 0 || d->teams_per_sm > 2)
+        return fail(NEST_ERR_INVALID_ARG, "teams_per_sm %d: need 0, 1 or 2", d->teams_per_sm);
+    if (d->teams_per_sm && d->x_halo <= 0)
+        return fail(NEST_ERR_INVALID_ARG, "teams_per_sm applies to the x ring (x_halo > 0) only");
     if (d->team_chunk < 0) return fail(NEST_ERR_INVALID_ARG, "team_chunk %d < 0", d->team_chunk);
     if (d->team_chunk > 0 && !(d->flags & NEST_F_BLOCKED))
         return fail(NEST_ERR_INVALID_ARG, "team_chunk needs NEST_F_BLOCKED");
@@ -108,22 +110,15 @@ static nest_status plan_core(const nest_desc* d, int64_t outer, int32_t K, int32
     if (outer < 0) return fail(NEST_ERR_INVALID_ARG, "outer iterations %lld < 0", (long long)outer);
     if (d->x_halo < 0) return fail(NEST_ERR_INVALID_ARG, "x_halo %d < 0", d->x_halo);
     if (d->x_halo > 0 && !spmv_window)
-        return fail(NEST_ERR_INVALID_ARG, "x_halo applies to the CSR SpMV only");
-    if ((d->flags & NEST_F_STAGED) && !spmv_window)
-        return fail(NEST_ERR_INVALID_ARG, "NEST_F_STAGED applies to the CSR SpMV only");
+        return fail(NEST_ERR_INVALID_ARG, "x_halo applies to the CSR SpMV only (nest_spmv_plan)");
     if (d->mode == NEST_MODE_TEAMS_GENERIC && !spmv_window)
         return fail(NEST_ERR_INVALID_ARG, "NEST_MODE_TEAMS_GENERIC applies to the CSR SpMV only");
     if ((d->flags & NEST_F_VEC_QUAD) && !spmv_window)
         return fail(NEST_ERR_INVALID_ARG, "NEST_F_VEC_QUAD applies to the CSR SpMV only");
     if ((d->flags & NEST_F_VEC_QUAD) && !(d->flags & NEST_F_VEC128))
         return fail(NEST_ERR_INVALID_ARG, "NEST_F_VEC_QUAD needs NEST_F_VEC128");
-    if ((d->flags & NEST_F_VEC128) && (d->flags & NEST_F_STAGED))
-        return fail(NEST_ERR_UNSUPPORTED, "NEST_F_VEC128 does not combine with NEST_F_STAGED");
     if ((d->flags & NEST_F_VEC_QUAD) && d->x_halo > 0)
         return fail(NEST_ERR_UNSUPPORTED, "x_halo takes scalar or pair loads (not NEST_F_VEC_QUAD)");
-    if ((d->flags & NEST_F_STAGED) && T < 128)
-        return fail(NEST_ERR_INVALID_ARG,
-                    "NEST_F_STAGED needs threads_per_team >= 128 (producer, 2 gather and >= 1 consumer warps)");
     if (K <= 0) K = 1;
     const int32_t S = d->simdlen;
     const bool smem_mode = d->mode == NEST_MODE_GENERIC_SMEM && S > 1;
@@ -144,48 +139,9 @@ static nest_status plan_core(const nest_desc* d, int64_t outer, int32_t K, int32
     const int64_t per_group = (U + K - 1) / K;
     const int64_t denom = (int64_t)q.groups * per_group;
     int64_t needed = (outer + denom - 1) / denom;
-    if (d->flags & NEST_F_STAGED) {
-        q.x_halo = d->x_halo;   // stage sizes and grid: plan_spmv_staged (needs nnz)
+    if (d->x_halo > 0) {
+        q.x_halo = d->x_halo;   // the x ring: sized by plan_spmv_ring (needs nnz)
         q.grid = d->num_teams;
-    } else if (d->x_halo > 0) {
-        // x window (spmv_xwin.cuh): ring of XW = 2R + 2H doubles, R = G*U*KB rows per
-        // chunk (even), H = x_halo rounded up to even; KB: the most rows per chunk
-        // whose ring still lets 2048 / T teams share an SM, else the fewest that fit.
-        const int64_t H = ((int64_t)d->x_halo + 1) & ~(int64_t)1;
-        const int64_t per_sm = kMaxThreadsPerSm / T > 0 ? kMaxThreadsPerSm / T : 1;
-        const int64_t budget = kSmemPerSm / per_sm - kSmemReservedPerBlock;
-        int64_t kb = 0, bytes = 0;
-        for (int64_t k = 16; k >= 1; k >>= 1) {
-            const int64_t R = (int64_t)q.groups * U * k;
-            const int64_t b = (2 * R + 2 * H) * 8 + 16 + q.smem_bytes;
-            if (R % 2 == 0 && b <= budget && b <= kMaxDynSmem) {
-                kb = k, bytes = b;
-                break;
-            }
-        }
-        for (int64_t k = 1; kb == 0 && k <= 16; k <<= 1) {
-            const int64_t R = (int64_t)q.groups * U * k;
-            const int64_t b = (2 * R + 2 * H) * 8 + 16 + q.smem_bytes;
-            if (R % 2 == 0 && b <= kMaxDynSmem) kb = k, bytes = b;
-        }
-        if (kb == 0)
-            return fail(NEST_ERR_UNSUPPORTED,
-                        "x_halo %d with %lld rows per batch needs more than %d B of shared memory",
-                        d->x_halo, (long long)q.groups * U, kMaxDynSmem);
-        const int64_t R = (int64_t)q.groups * U * kb;
-        q.x_halo = (int32_t)H;
-        q.kb = (int32_t)kb;
-        q.xw = (int32_t)(2 * R + 2 * H);
-        q.smem_bytes = (int32_t)bytes;
-        const int64_t chunks = (outer + R - 1) / R;
-        if (d->num_teams > 0) {
-            q.grid = d->num_teams;
-        } else {
-            int64_t resident = 0;
-            nest_status s = resident_blocks(T, q.smem_bytes, &resident);
-            if (s != NEST_OK) return s;
-            q.grid = (int32_t)(chunks < resident ? (chunks > 0 ? chunks : 1) : resident);
-        }
     } else if (d->num_teams > 0) {
         q.grid = d->num_teams;
     } else if ((d->flags & (NEST_F_PERSISTENT_GRID | NEST_F_BLOCKED)) || q.fallback) {
@@ -318,12 +274,7 @@ NEST_API const char* nest_status_str(nest_status s) {
 
 NEST_API const char* nest_last_error(void) { return nest::g_err; }
 
-NEST_API nest_status nest_plan(const nest_desc* desc, int64_t outer_iters, int32_t payload_bytes,
-                               nest_plan_info* out) {
-    if (!out) return fail(NEST_ERR_INVALID_ARG, "out is NULL");
-    Plan p;
-    nest_status s = make_plan_fixed(desc, outer_iters, 1, payload_bytes, &p, true);
-    if (s != NEST_OK) return s;
+static void fill_plan_info(const Plan& p, int32_t kernel, int32_t index_bits, nest_plan_info* out) {
     out->grid = p.grid;
     out->block = p.block;
     out->groups_per_team = p.groups;
@@ -332,6 +283,91 @@ NEST_API nest_status nest_plan(const nest_desc* desc, int64_t outer_iters, int32
     out->uses_global_fallback = p.fallback;
     out->outer_unroll = p.unroll;
     out->smem_bytes = p.smem_bytes;
+    out->kernel = kernel;
+    out->index_bits = index_bits;
+    out->ring_segments = p.ring_nseg;
+    out->ring_row_slots = p.ring_nrp;
+    out->chunk = (p.flags & NEST_F_BLOCKED) || p.x_halo > 0 ? p.chunk : 0;
+}
+
+NEST_API nest_status nest_plan(const nest_desc* desc, int64_t outer_iters, int32_t payload_bytes,
+                               nest_plan_info* out) {
+    if (!out) return fail(NEST_ERR_INVALID_ARG, "out is NULL");
+    Plan p;
+    nest_status s = make_plan_fixed(desc, outer_iters, 1, payload_bytes, &p, false);
+    if (s != NEST_OK) return s;
+    fill_plan_info(p, NEST_KERNEL_NEST, 64, out);
+    return NEST_OK;
+}
+
+// The plan the CSR SpMV launches for this matrix shape (a1 for a8): the
+// descriptor's geometry, the variant's own sizing (x ring, teams-generic), and
+// the generic payload of the body that actually runs -- so the reported
+// fallback is the kernel's (engine.cuh group_slot follows the plan).
+static nest_status spmv_plan(const nest_desc* desc, int64_t nrows, int64_t ncols, int64_t nnz, Plan* p,
+                             int32_t* kernel, int32_t* index_bits) {
+    if (nrows < 0 || ncols < 0 || nnz < 0)
+        return fail(NEST_ERR_INVALID_ARG, "negative extent (nrows %lld, ncols %lld, nnz %lld)",
+                    (long long)nrows, (long long)ncols, (long long)nnz);
+    if (ncols > INT32_MAX) return fail(NEST_ERR_INVALID_ARG, "ncols exceeds int32 column indices");
+    nest_status s = make_plan(desc, nrows, 1, spmv_payload, p, true);
+    if (s != NEST_OK) return s;
+    if (desc->mode == NEST_MODE_TEAMS_GENERIC) {
+        if ((p->flags & (NEST_F_VEC128 | NEST_F_BLOCKED)) || p->x_halo > 0)
+            return fail(NEST_ERR_UNSUPPORTED, "NEST_MODE_TEAMS_GENERIC takes no SpMV variant flags");
+        if (desc->num_teams <= 0) {
+            int64_t resident = 0;
+            if ((s = resident_blocks(p->block + 32, 0, &resident)) != NEST_OK) return s;
+            p->grid = (int32_t)std::max<int64_t>(1, std::min(nrows, resident));
+        }
+        *kernel = NEST_KERNEL_TEAMS_GENERIC;
+        *index_bits = 64;
+        return NEST_OK;
+    }
+    if (p->x_halo > 0) {
+        *kernel = NEST_KERNEL_XRING;
+        *index_bits = nnz < ((int64_t)1 << 31) - 8 && nrows < ((int64_t)1 << 31) - 8 ? 32 : 64;
+        return plan_spmv_ring(p, nrows, nnz, desc->num_teams, desc->teams_per_sm);
+    }
+    *kernel = NEST_KERNEL_NEST;
+    const int32_t payload = spmv_body_payload(*p, nnz);
+    if (payload != p->payload_bytes && (s = make_plan_fixed(desc, nrows, 1, payload, p, true)) != NEST_OK) return s;
+    *index_bits = spmv_index32(*p, nnz) ? 32 : 64;
+    return NEST_OK;
+}
+
+NEST_API nest_status nest_spmv_plan(const nest_desc* desc, int64_t nrows, int64_t ncols, int64_t nnz,
+                                    nest_plan_info* out) {
+    if (!out) return fail(NEST_ERR_INVALID_ARG, "out is NULL");
+    Plan p;
+    int32_t kernel = 0, bits = 0;
+    nest_status s = spmv_plan(desc, nrows, ncols, nnz, &p, &kernel, &bits);
+    if (s != NEST_OK) return s;
+    fill_plan_info(p, kernel, bits, out);
+    return NEST_OK;
+}
+
+// Launch a planned SpMV on rows [0, nrows) of the given arrays (rowptr entries
+// are absolute offsets into colind/val).
+static nest_status spmv_launch(const Plan& p, int32_t kernel, int64_t nrows, int64_t ncols, int64_t nnz,
+                               const int64_t* rowptr, const int32_t* colind, const double* val, const double* x,
+                               double* y, unsigned char* fb, cudaStream_t st) {
+    if (kernel == NEST_KERNEL_TEAMS_GENERIC) return launch_spmv_teams_generic(p, nrows, rowptr, colind, val, x, y, st);
+    if (kernel == NEST_KERNEL_XRING) return launch_spmv_ring(p, nrows, ncols, nnz, rowptr, colind, val, x, y, fb, st);
+    return launch_spmv(p, (p.flags & NEST_F_STREAM_HINTS) != 0, nrows, rowptr, colind, val, x, y, fb, st, nnz);
+}
+
+// Alignment the variants need (checked before any launch).
+static nest_status spmv_alignment(const Plan& p, int32_t kernel, const int64_t* rowptr, const int32_t* colind,
+                                  const double* val, const double* x) {
+    if (reinterpret_cast<uintptr_t>(rowptr) & 7) return fail(NEST_ERR_INVALID_ARG, "rowptr must be 8-byte aligned");
+    if ((p.flags & NEST_F_VEC128) &&
+        ((reinterpret_cast<uintptr_t>(val) & 15) ||
+         (reinterpret_cast<uintptr_t>(colind) & ((p.flags & NEST_F_VEC_QUAD) ? 15 : 7))))
+        return fail(NEST_ERR_UNSUPPORTED, "NEST_F_VEC128 needs 16-byte aligned val and %d-byte aligned colind",
+                    (p.flags & NEST_F_VEC_QUAD) ? 16 : 8);
+    if (kernel == NEST_KERNEL_XRING && (reinterpret_cast<uintptr_t>(x) & 15))
+        return fail(NEST_ERR_UNSUPPORTED, "x_halo needs 16-byte aligned x (bulk copies of x segments)");
     return NEST_OK;
 }
 
@@ -339,48 +375,17 @@ NEST_API nest_status nest_spmv_csr_f64(const nest_desc* desc, int64_t nrows, int
                                        int64_t nnz, const int64_t* rowptr, const int32_t* colind,
                                        const double* val, const double* x, double* y,
                                        void* stream) {
-    if (nrows < 0 || ncols < 0 || nnz < 0)
-        return fail(NEST_ERR_INVALID_ARG, "negative extent (nrows %lld, ncols %lld, nnz %lld)",
-                    (long long)nrows, (long long)ncols, (long long)nnz);
-    if (ncols > INT32_MAX) return fail(NEST_ERR_INVALID_ARG, "ncols exceeds int32 column indices");
     Plan p;
-    nest_status s = make_plan(desc, nrows, 1, spmv_payload, &p, true);
+    int32_t kernel = 0, bits = 0;
+    nest_status s = spmv_plan(desc, nrows, ncols, nnz, &p, &kernel, &bits);
     if (s != NEST_OK) return s;
     if (nrows == 0) return NEST_OK;
     if (!rowptr || !y) return fail(NEST_ERR_INVALID_ARG, "rowptr/y is NULL");
     if (nnz > 0 && (!colind || !val || !x)) return fail(NEST_ERR_INVALID_ARG, "colind/val/x is NULL");
-    if (desc->mode == NEST_MODE_TEAMS_GENERIC) {
-        if (p.flags & (NEST_F_STAGED | NEST_F_VEC128 | NEST_F_BLOCKED) || p.x_halo > 0)
-            return fail(NEST_ERR_UNSUPPORTED, "NEST_MODE_TEAMS_GENERIC takes no SpMV variant flags");
-        if (desc->num_teams <= 0) {
-            int64_t resident = 0;
-            if ((s = resident_blocks(p.block + 32, 0, &resident)) != NEST_OK) return s;
-            p.grid = (int32_t)(nrows < resident ? nrows : resident);
-        }
-        return launch_spmv_teams_generic(p, nrows, rowptr, colind, val, x, y, as_stream(stream));
-    }
-    const bool staged = (p.flags & NEST_F_STAGED) != 0;
-    if (staged && (s = plan_spmv_staged(&p, nrows, nnz, desc->sharing_bytes ? desc->sharing_bytes : kDefaultSharing)) != NEST_OK)
-        return s;
-    if (staged && ((reinterpret_cast<uintptr_t>(colind) | reinterpret_cast<uintptr_t>(val) |
-                    reinterpret_cast<uintptr_t>(x)) & 15))
-        return fail(NEST_ERR_UNSUPPORTED, "NEST_F_STAGED needs 16-byte aligned colind, val and x");
+    if ((s = spmv_alignment(p, kernel, rowptr, colind, val, x)) != NEST_OK) return s;
     unsigned char* fb = nullptr;
     if ((s = prepare_fallback(p, &fb, stream)) != NEST_OK) return s;
-    if ((p.flags & NEST_F_VEC128) &&
-        ((reinterpret_cast<uintptr_t>(val) & 15) ||
-         (reinterpret_cast<uintptr_t>(colind) & ((p.flags & NEST_F_VEC_QUAD) ? 15 : 7))))
-        return fail(NEST_ERR_UNSUPPORTED, "NEST_F_VEC128 needs 16-byte aligned val and %d-byte aligned colind",
-                    (p.flags & NEST_F_VEC_QUAD) ? 16 : 8);
-    if (staged) return launch_spmv_staged(p, nrows, ncols, nnz, rowptr, colind, val, x, y, fb, as_stream(stream));
-    if (p.x_halo > 0) {
-        if (reinterpret_cast<uintptr_t>(x) & 15) return fail(NEST_ERR_UNSUPPORTED, "x_halo needs 16-byte aligned x");
-        if ((p.flags & NEST_F_VEC128) && (nnz >= ((int64_t)1 << 31) - 8 || nrows >= ((int64_t)1 << 31) - 8))
-            return fail(NEST_ERR_UNSUPPORTED, "x_halo with NEST_F_VEC128 needs nnz, nrows < 2^31");
-        return launch_spmv_xwin(p, nrows, ncols, nnz, rowptr, colind, val, x, y, fb, as_stream(stream));
-    }
-    return launch_spmv(p, (p.flags & NEST_F_STREAM_HINTS) != 0, nrows, rowptr, colind, val, x, y, fb,
-                       as_stream(stream), nnz);
+    return spmv_launch(p, kernel, nrows, ncols, nnz, rowptr, colind, val, x, y, fb, as_stream(stream));
 }
 
 static size_t align256(size_t b) { return (b + 255) & ~(size_t)255; }
@@ -454,7 +459,7 @@ static nest_status spmv_hostio_pipelined(const nest_desc* desc, int nchunks, int
                                          int64_t ncols, int64_t nnz, const int64_t* h_rowptr,
                                          const int32_t* h_colind, const double* h_val, const double* h_x,
                                          double* h_y, int64_t* d_rowptr, int32_t* d_col, double* d_val,
-                                         double* d_x, double* d_y, unsigned char* fb, cudaStream_t st) {
+                                         double* d_x, double* d_y, cudaStream_t st) {
     // chunk c = rows [r[c], r[c+1]) with nonzeros [h_rowptr[r[c]], h_rowptr[r[c+1]]);
     // boundaries at the rows where the nonzero count crosses c * nnz / nchunks
     int64_t r[kHostioMaxChunks + 1];
@@ -508,9 +513,12 @@ static nest_status spmv_hostio_pipelined(const nest_desc* desc, int nchunks, int
         if ((e = cudaStreamWaitEvent(st, ev_in[j], 0))) return cuda_fail(e, "hostio wait");
         if (rows > 0) {
             Plan p;
-            if ((s = make_plan(desc, rows, 1, spmv_payload, &p, true)) != NEST_OK) return s;
-            if ((s = launch_spmv(p, (p.flags & NEST_F_STREAM_HINTS) != 0, rows, d_rowptr + r[c], d_col, d_val,
-                                 d_x, d_y + r[c], fb, st, nnz)) != NEST_OK)
+            int32_t kernel = 0, bits = 0;
+            unsigned char* fb = nullptr;
+            if ((s = spmv_plan(desc, rows, ncols, nnz, &p, &kernel, &bits)) != NEST_OK ||
+                (s = prepare_fallback(p, &fb, st)) != NEST_OK ||
+                (s = spmv_launch(p, kernel, rows, ncols, nnz, d_rowptr + r[c], d_col, d_val, d_x, d_y + r[c], fb, st)) !=
+                    NEST_OK)
                 return s;
         }
         if ((e = cudaEventRecord(ev_k[c], st)) || (e = cudaStreamWaitEvent(h->d2h, ev_k[c], 0)))
@@ -529,16 +537,18 @@ NEST_API nest_status nest_spmv_csr_f64_hostio(const nest_desc* desc, int64_t nro
                                               const int32_t* h_colind, const double* h_val,
                                               const double* h_x, double* h_y, void* d_workspace,
                                               size_t workspace_bytes, void* stream) {
-    if (nrows < 0 || ncols < 0 || nnz < 0) return fail(NEST_ERR_INVALID_ARG, "negative extent");
     Plan p;
-    nest_status s = make_plan(desc, nrows, 1, spmv_payload, &p, true);
+    int32_t kernel = 0, bits = 0;
+    nest_status s = spmv_plan(desc, nrows, ncols, nnz, &p, &kernel, &bits);
     if (s != NEST_OK) return s;
     if (nrows == 0) return NEST_OK;
-    if (desc->mode == NEST_MODE_TEAMS_GENERIC)
+    if (kernel == NEST_KERNEL_TEAMS_GENERIC)
         return fail(NEST_ERR_UNSUPPORTED, "nest_spmv_csr_f64_hostio: use nest_spmv_csr_f64 for NEST_MODE_TEAMS_GENERIC");
     const size_t need = nest_spmv_hostio_workspace_bytes(nrows, ncols, nnz);
     if (!d_workspace || workspace_bytes < need)
         return fail(NEST_ERR_INVALID_ARG, "workspace %zu bytes < %zu", workspace_bytes, need);
+    if (reinterpret_cast<uintptr_t>(d_workspace) & 255)
+        return fail(NEST_ERR_INVALID_ARG, "workspace must be 256-byte aligned");
     if (!h_rowptr || !h_y || (nnz > 0 && (!h_colind || !h_val || !h_x)))
         return fail(NEST_ERR_INVALID_ARG, "host buffer is NULL");
     if (h_rowptr[0] != 0 || h_rowptr[nrows] != nnz)
@@ -554,29 +564,20 @@ NEST_API nest_status nest_spmv_csr_f64_hostio(const nest_desc* desc, int64_t nro
     double* d_x = reinterpret_cast<double*>(w);
     w += align256((size_t)ncols * 8);
     double* d_y = reinterpret_cast<double*>(w);
-    const bool staged = (p.flags & NEST_F_STAGED) != 0;
-    if (staged && (s = plan_spmv_staged(&p, nrows, nnz, desc->sharing_bytes ? desc->sharing_bytes : kDefaultSharing)) != NEST_OK)
-        return s;
-    if (p.x_halo > 0 && (p.flags & NEST_F_VEC128) && (nnz >= ((int64_t)1 << 31) - 8 || nrows >= ((int64_t)1 << 31) - 8))
-        return fail(NEST_ERR_UNSUPPORTED, "x_halo with NEST_F_VEC128 needs nnz, nrows < 2^31");
-    unsigned char* fb = nullptr;
-    if ((s = prepare_fallback(p, &fb, stream)) != NEST_OK) return s;
     cudaStream_t st = as_stream(stream);
-    cudaError_t e;
-    const int nchunks = staged || p.x_halo > 0 ? 1 : hostio_chunks(nnz);
+    const int nchunks = hostio_chunks(nnz);
     if (nchunks > 1)
         return spmv_hostio_pipelined(desc, nchunks, nrows, ncols, nnz, h_rowptr, h_colind, h_val, h_x, h_y,
-                                     d_rowptr, d_col, d_val, d_x, d_y, fb, st);
+                                     d_rowptr, d_col, d_val, d_x, d_y, st);
+    unsigned char* fb = nullptr;
+    if ((s = prepare_fallback(p, &fb, stream)) != NEST_OK) return s;
+    cudaError_t e;
     if ((e = cudaMemcpyAsync(d_rowptr, h_rowptr, (size_t)(nrows + 1) * 8, cudaMemcpyHostToDevice, st)) ||
         (nnz && (e = cudaMemcpyAsync(d_col, h_colind, (size_t)nnz * 4, cudaMemcpyHostToDevice, st))) ||
         (nnz && (e = cudaMemcpyAsync(d_val, h_val, (size_t)nnz * 8, cudaMemcpyHostToDevice, st))) ||
         (ncols && (e = cudaMemcpyAsync(d_x, h_x, (size_t)ncols * 8, cudaMemcpyHostToDevice, st))))
         return cuda_fail(e, "host->device copy");
-    s = staged ? launch_spmv_staged(p, nrows, ncols, nnz, d_rowptr, d_col, d_val, d_x, d_y, fb, st)
-        : p.x_halo > 0 ? launch_spmv_xwin(p, nrows, ncols, nnz, d_rowptr, d_col, d_val, d_x, d_y, fb, st)
-                     : launch_spmv(p, (p.flags & NEST_F_STREAM_HINTS) != 0, nrows, d_rowptr, d_col, d_val,
-                                   d_x, d_y, fb, st, nnz);
-    if (s != NEST_OK) return s;
+    if ((s = spmv_launch(p, kernel, nrows, ncols, nnz, d_rowptr, d_col, d_val, d_x, d_y, fb, st)) != NEST_OK) return s;
     if ((e = cudaMemcpyAsync(h_y, d_y, (size_t)nrows * 8, cudaMemcpyDeviceToHost, st)))
         return cuda_fail(e, "device->host copy");
     return NEST_OK;
@@ -667,9 +668,7 @@ NEST_API nest_status nest_util_l2_flush(void* buf, size_t bytes, void* stream) {
     const size_t n16 = bytes / 16;
     if (n16 == 0) return NEST_OK;
     l2_flush_kernel<<<1184, 512, 0, as_stream(stream)>>>(static_cast<uint4*>(buf), n16, salt++);
-    const char* ce = std::getenv("NEST_FLUSH_CLEAN");   // 0: write phase only (A/B experiments)
-    if (!ce || std::atoi(ce) != 0)
-        l2_clean_kernel<<<1184, 512, 0, as_stream(stream)>>>(static_cast<const uint4*>(buf), n16 / 2, nullptr);
+    l2_clean_kernel<<<1184, 512, 0, as_stream(stream)>>>(static_cast<const uint4*>(buf), n16 / 2, nullptr);
     const cudaError_t e = cudaGetLastError();
     return e == cudaSuccess ? NEST_OK : cuda_fail(e, "l2_flush launch");
 }

@@ -146,7 +146,7 @@ struct XPeer {
 // sparse_matvec: outer loop over rows on "teams distribute
 // parallel for", inner loop over the row's nonzeros on "simd".  The product is
 // reduced in-group (R2) instead of the paper's atomic update.
-template <bool HINTS, bool PIPE = false, class I = int64_t, class XA = XLocal>
+template <bool HINTS, class I = int64_t, class XA = XLocal>
 struct SpmvBody {
     using Acc = double;
     using OuterIndex = I;   // launcher: I = int32_t only when spmv_index32()
@@ -165,39 +165,12 @@ struct SpmvBody {
     const int64_t* rowptr;
     const int32_t* col;
     const double* val;
-    XA x;   // x access (XLocal: x[c]; XPeer: the owner rank's slice)
+    XA x;   // x access (XLocal: x[c]; XPeer: the owner rank's slice; XRing: the staged window)
     double* y;
-    // L2 prefetch of the team's upcoming nonzeros (blocked schedule): the team
-    // leader prefetches [base + pf_ahead, base + pf_ahead + pf_len) of colind and
-    // val with bulk L2 prefetches (TMA engine), so the groups' loads hit L2.
     int64_t nnz = 0;
-    int64_t pf_ahead = 0;
-    int64_t pf_len = 0;
-    static constexpr bool kL2Hint = true;
 
-    __device__ __forceinline__ void team_hint(const Loop& L) const {
-        if (pf_len <= 0) return;
-        int64_t b = (L.base + pf_ahead) & ~(int64_t)3;
-        int64_t e = (b + pf_len + 3) & ~(int64_t)3;
-        const int64_t lim = nnz & ~(int64_t)3;
-        if (e > lim) e = lim;
-        if (e <= b) return;
-        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;\n" ::"l"(col + b), "r"((uint32_t)((e - b) * 4)) : "memory");
-        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;\n" ::"l"(val + b), "r"((uint32_t)((e - b) * 8)) : "memory");
-    }
-
-    // loop-bound pipeline (engine.cuh): rowptr[i], rowptr[i+1] -> 16 shared bytes
-    static constexpr bool kRowptrPipe = PIPE;
-    __device__ __forceinline__ void pipe_issue(int64_t i, unsigned char* slot) const {
-        const unsigned s0 = (unsigned)__cvta_generic_to_shared(slot);
-        asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(s0), "l"(rowptr + i) : "memory");
-        asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(s0 + 8), "l"(rowptr + i + 1) : "memory");
-    }
-    __device__ __forceinline__ Loop pipe_loop(int64_t i, const unsigned char* slot, Step& st) const {
-        const int64_t* v = reinterpret_cast<const int64_t*>(slot);
-        st.i = (I)i;
-        return Loop{(I)(v[1] - v[0]), (I)v[0]};
-    }
+    // the simd loop of the row [b, e): the loop state the sequential code computes
+    static __device__ __forceinline__ Loop loop_of(int64_t b, int64_t e) { return Loop{(I)(e - b), (I)b}; }
 
     static __device__ __forceinline__ int steps(const SpmvBody&) { return 1; }
     static __device__ __forceinline__ void team_begin(TeamShared&) {}
@@ -205,9 +178,7 @@ struct SpmvBody {
 
     __device__ __forceinline__ Loop prologue(int64_t i, int, Step& st, bool, TeamShared&) const {
         st.i = (I)i;
-        const I b = (I)__ldg(rowptr + i);
-        const I e = (I)__ldg(rowptr + i + 1);
-        return Loop{e - b, b};
+        return loop_of(__ldg(rowptr + i), __ldg(rowptr + i + 1));
     }
     template <int OP>
     __device__ __forceinline__ double accum(const Loop& L, I j, double acc) const {
@@ -287,12 +258,15 @@ struct SpmvVecBody {
     static __device__ __forceinline__ void team_begin(TeamShared&) {}
     static __device__ __forceinline__ void team_end(const SpmvVecBody&, TeamShared&) {}
 
-    __device__ __forceinline__ Loop prologue(int64_t i, int, Step& st, bool, TeamShared&) const {
-        st.i = (I)i;
-        const I b = (I)__ldg(rowptr + i);
-        const I e = (I)__ldg(rowptr + i + 1);
+    // the simd loop of the row [b, e): tuples covering it, from the aligned tuple holding b
+    static __device__ __forceinline__ Loop loop_of(int64_t b64, int64_t e64) {
+        const I b = (I)b64, e = (I)e64;
         constexpr int kLog = V == 2 ? 1 : 2;
         return Loop{b, e > b ? (int32_t)(((e + V - 1) >> kLog) - (b >> kLog)) : 0, (int32_t)(e - b)};
+    }
+    __device__ __forceinline__ Loop prologue(int64_t i, int, Step& st, bool, TeamShared&) const {
+        st.i = (I)i;
+        return loop_of(__ldg(rowptr + i), __ldg(rowptr + i + 1));
     }
     // the tuple starting at entry k0: 128-bit loads, scalar at the end of the arrays
     __device__ __forceinline__ void load_tuple(I k0, int32_t (&c)[V], double (&v)[V]) const {

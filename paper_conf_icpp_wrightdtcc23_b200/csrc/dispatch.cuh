@@ -5,8 +5,6 @@
 // compile-time variant, so the hot loop has no indirect call.
 #pragma once
 
-#include <cstdlib>
-
 #include "bodies/bodies.cuh"
 #include "internal.h"
 
@@ -34,24 +32,13 @@ nest_status launch_one(const Plan& p, const Body& body, unsigned char* fb, cudaS
         return fail(NEST_ERR_UNSUPPORTED,
                     "threads_per_team %d exceeds this variant's limit of %d (registers); use a smaller team or "
                     "outer_unroll", p.block, max_threads);
-    // L1 / shared-memory split (percent of the maximum shared carve-out; -1: driver's choice)
-    static const int carveout = [] {
-        const char* e = std::getenv("NEST_CARVEOUT");
-        return e ? std::atoi(e) : -1;
-    }();
-    static bool carveout_set = false;
-    if (carveout >= 0 && !carveout_set) {
-        const cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, carveout);
-        if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(carveout)");
-        carveout_set = true;
-    }
     if (p.smem_bytes > 48 * 1024) {
         const cudaError_t e = cudaFuncSetAttribute(kern,
                                                    cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem_bytes);
         if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(max dynamic smem)");
     }
     kern<<<p.grid, p.block, p.smem_bytes, st>>>(
-        body, p.outer, p.slot_bytes, fb, (p.flags & NEST_F_BLOCKED) ? p.chunk : 0, p.pipe_off);
+        body, p.outer, p.slot_bytes, fb, (p.flags & NEST_F_BLOCKED) ? p.chunk : 0);
     const cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e, "kernel launch");
     return NEST_OK;

@@ -77,9 +77,11 @@ NEST_API nest_status nest_spmv_csr_f64_dist(const nest_desc* desc, nest_comm* c,
     const int64_t xchunk = (ncols_global + c->nranks - 1) / c->nranks;
     if (xchunk > 0 && (!x_local || !x_full)) return fail(NEST_ERR_INVALID_ARG, "x_local/x_full is NULL");
     // validate the local launch before enqueuing the collective (no side effects on error)
-    Plan p;
-    nest_status s = make_plan(desc, nrows_local, 1, spmv_payload, &p, true);
+    nest_plan_info info;
+    nest_status s = nest_spmv_plan(desc, nrows_local, ncols_global, nnz_local, &info);
     if (s != NEST_OK) return s;
+    if (nrows_local > 0 && (!rowptr_local || !y_local)) return fail(NEST_ERR_INVALID_ARG, "rowptr/y is NULL");
+    if (nnz_local > 0 && (!colind || !val)) return fail(NEST_ERR_INVALID_ARG, "colind/val is NULL");
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
     if (xchunk > 0) {
         const ncclResult_t r =

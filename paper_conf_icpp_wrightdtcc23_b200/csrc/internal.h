@@ -28,14 +28,14 @@ struct Plan {
     uint32_t flags = 0;
     int64_t outer = 0;
     int64_t chunk = 0;     // NEST_F_BLOCKED: outer iterations per team chunk (a multiple of G)
-    int32_t x_halo = 0;    // SpMV x window half-width (0 = none)
-    int32_t kb = 1;        // x window: batches of U rows per group per chunk
-    // NEST_F_STAGED pipeline (spmv_staged.cuh)
-    int32_t xw = 0;        // x ring capacity in doubles (even; 0 = no window)
-    int32_t nb = 0;        // stage capacity in nonzeros
-    int32_t ns = 0;        // stages in flight
-    int32_t rmax = 0;      // rows per chunk at most
-    int32_t pipe_off = -1; // nest_kernel loop-bound pipeline ring offset in dynamic smem (-1 = off)
+    int32_t x_halo = 0;    // SpMV x ring: window half-width H (0 = no ring)
+    // x ring (device/spmv_ring.cuh), planned by plan_spmv_ring
+    int32_t ring_nseg = 0;       // x segment slots
+    int32_t ring_nrp = 0;        // row-bound stages per consumer warp (prefetch depth)
+    int32_t ring_rp_stride = 0;  // int64 entries per row-bound stage
+    int32_t ring_kb = 1;         // rows per group per round (= outer_unroll)
+    int32_t ring_tps = 0;        // teams per SM the ring is sized for
+    int64_t per_team = 0;        // rows per team
 };
 
 // 32-bit row / nonzero indices (and 32-bit outer-loop cursors, engine.cuh
@@ -77,14 +77,14 @@ int32_t laplace_payload(int32_t U);
 nest_status launch_spmv(const Plan& p, bool hints, int64_t nrows, const int64_t* rowptr,
                         const int32_t* col, const double* val, const double* x, double* y,
                         unsigned char* fb, cudaStream_t st, int64_t nnz);
-nest_status launch_spmv_xwin(const Plan& p, int64_t nrows, int64_t ncols, int64_t nnz, const int64_t* rowptr,
+// x ring (x_halo > 0): finish the plan (ring sizes, teams, payload of the launched
+// body) from the matrix shape, and launch.
+nest_status plan_spmv_ring(Plan* p, int64_t nrows, int64_t nnz, int32_t num_teams, int32_t teams_per_sm);
+nest_status launch_spmv_ring(const Plan& p, int64_t nrows, int64_t ncols, int64_t nnz, const int64_t* rowptr,
                              const int32_t* col, const double* val, const double* x, double* y,
                              unsigned char* fb, cudaStream_t st);
-// NEST_F_STAGED: finish the plan from the matrix shape (stage sizes, grid) and launch.
-nest_status plan_spmv_staged(Plan* p, int64_t nrows, int64_t nnz, int32_t sharing_bytes);
-nest_status launch_spmv_staged(const Plan& p, int64_t nrows, int64_t ncols, int64_t nnz,
-                               const int64_t* rowptr, const int32_t* col, const double* val,
-                               const double* x, double* y, unsigned char* fb, cudaStream_t st);
+// payload (bytes of one generic slot) of the body launch_spmv runs for plan p
+int32_t spmv_body_payload(const Plan& p, int64_t nnz);
 nest_status resident_blocks(int32_t T, int32_t smem, int64_t* out);
 nest_status launch_batched(const Plan& p, int64_t batch, int32_t m, int32_t n, const float* A,
                            const float* x, float* y, unsigned char* fb, cudaStream_t st);

@@ -19,6 +19,7 @@ struct RegionArgs {
     int32_t kind, simdlen, mode, slot_bytes;
     int64_t n_outer, chunk;     // outer iterations; team chunk (0 = cyclic)
     int64_t fb_offset;          // byte offset of this region's global fallback
+    int32_t use_fb;             // the region's payload exceeds its slot
     int64_t n[3];
     const void* in[4];
     void* out[2];
@@ -33,7 +34,7 @@ struct Program {
 // kernel's register allocation is the largest region's, not their sum.
 template <int S, int MODE, class Body>
 __device__ __noinline__ void region_call(const Body b, const RegionArgs& R, unsigned char* fb, unsigned char* smem) {
-    parallel_region<S, MODE, RED_SUM, 1>(b, R.n_outer, R.slot_bytes, fb, R.chunk, -1, smem);
+    parallel_region<S, MODE, RED_SUM, 1>(b, R.n_outer, R.slot_bytes, fb, R.chunk, smem);
 }
 
 template <int S, class Body>
@@ -73,10 +74,10 @@ __global__ void __launch_bounds__(1024, 1) region_program_kernel(const Program p
     for (int k = 0; k < NEST_MAX_REGIONS; ++k) {
         if (k >= prog.count) break;
         const RegionArgs& R = prog.r[k];
-        unsigned char* fb = gfallback ? gfallback + R.fb_offset : nullptr;
+        unsigned char* fb = R.use_fb ? gfallback + R.fb_offset : nullptr;
         switch (R.kind) {
             case NEST_REGION_SPMV_CSR_F64: {
-                SpmvBody<false, false, int64_t> b{static_cast<const int64_t*>(R.in[0]),
+                SpmvBody<false, int64_t> b{static_cast<const int64_t*>(R.in[0]),
                                                   static_cast<const int32_t*>(R.in[1]),
                                                   static_cast<const double*>(R.in[2]),
                                                   static_cast<const double*>(R.in[3]), static_cast<double*>(R.out[0])};
@@ -181,8 +182,8 @@ NEST_API nest_status nest_region_program(const nest_desc* desc, const nest_regio
             if (R.chunk == 0) R.chunk = G;
         }
         R.fb_offset = fb_bytes;
-        if (R.mode == NEST_MODE_GENERIC_SMEM && payload > R.slot_bytes)
-            fb_bytes += grid * G * payload;
+        R.use_fb = R.mode == NEST_MODE_GENERIC_SMEM && payload > R.slot_bytes;
+        if (R.use_fb) fb_bytes += grid * G * payload;
     }
     unsigned char* fb = nullptr;
     if (fb_bytes > 0 && (s = fallback_scratch((size_t)fb_bytes, &fb, stream)) != NEST_OK) return s;

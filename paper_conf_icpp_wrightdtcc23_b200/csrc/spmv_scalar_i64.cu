@@ -9,7 +9,7 @@ nest_status spmv_dispatch(const Plan& p, const Body& body, unsigned char* fb, cu
     return dispatch(p, body, fb, st);
 }
 
-template nest_status spmv_dispatch<SpmvBody<false, false, int64_t>>(const Plan&, const SpmvBody<false, false, int64_t>&, unsigned char*, cudaStream_t);
-template nest_status spmv_dispatch<SpmvBody<true, false, int64_t>>(const Plan&, const SpmvBody<true, false, int64_t>&, unsigned char*, cudaStream_t);
+template nest_status spmv_dispatch<SpmvBody<false, int64_t>>(const Plan&, const SpmvBody<false, int64_t>&, unsigned char*, cudaStream_t);
+template nest_status spmv_dispatch<SpmvBody<true, int64_t>>(const Plan&, const SpmvBody<true, int64_t>&, unsigned char*, cudaStream_t);
 
 }  // namespace nest

@@ -32,6 +32,16 @@ struct nest_xpeer {
 
 namespace nest {
 
+template <class Body>
+static int32_t xpeer_payload(int32_t U) {
+    switch (U) {
+        case 1: return payload_bytes<Body, 1>();
+        case 2: return payload_bytes<Body, 2>();
+        case 4: return payload_bytes<Body, 4>();
+    }
+    return -1;
+}
+
 nest_status launch_spmv_xpeer_vec(const Plan& p, const int64_t* rowptr, const int32_t* col, const double* val,
                                   XPeer xa, double* y, unsigned char* fb, cudaStream_t st, int64_t nnz);
 
@@ -232,7 +242,7 @@ NEST_API nest_status nest_spmv_csr_f64_xpeer(const nest_desc* desc, nest_xpeer* 
     Plan p;
     nest_status s = make_plan(desc, nrows_local, 1, spmv_payload, &p, true);
     if (s != NEST_OK) return s;
-    if (desc->mode == NEST_MODE_TEAMS_GENERIC || (p.flags & (NEST_F_STAGED | NEST_F_VEC_QUAD)) || p.x_halo > 0)
+    if (desc->mode == NEST_MODE_TEAMS_GENERIC || (p.flags & NEST_F_VEC_QUAD) || p.x_halo > 0)
         return fail(NEST_ERR_UNSUPPORTED,
                     "nest_spmv_csr_f64_xpeer: cyclic/blocked schedules with scalar or pair loads only");
     if (nrows_local > 0 && (!rowptr || !y)) return fail(NEST_ERR_INVALID_ARG, "rowptr/y is NULL");
@@ -240,6 +250,11 @@ NEST_API nest_status nest_spmv_csr_f64_xpeer(const nest_desc* desc, nest_xpeer* 
     const bool vec = (p.flags & NEST_F_VEC128) != 0;
     const bool i32 = spmv_index32(p, nnz);
     if (vec && !i32) return fail(NEST_ERR_UNSUPPORTED, "NEST_F_VEC128 (xpeer) needs nnz_local < 2^31, nrows_local < 2^30");
+    // the generic payload of the body that runs (the kernel follows the plan's fallback decision)
+    const int32_t payload = vec ? xpeer_payload<SpmvVecBody<false, 2, int32_t, XPeer>>(p.unroll)
+                                : xpeer_payload<SpmvBody<false, int64_t, XPeer>>(p.unroll);
+    if (payload != p.payload_bytes && (s = make_plan_fixed(desc, nrows_local, 1, payload, &p, true)) != NEST_OK)
+        return s;
     if (vec && ((reinterpret_cast<uintptr_t>(val) & 15) || (reinterpret_cast<uintptr_t>(colind) & 7)))
         return fail(NEST_ERR_UNSUPPORTED, "NEST_F_VEC128 needs 16-byte aligned val and 8-byte aligned colind");
     unsigned char* fb = nullptr;
@@ -253,7 +268,7 @@ NEST_API nest_status nest_spmv_csr_f64_xpeer(const nest_desc* desc, nest_xpeer* 
         if (vec) {
             s = launch_spmv_xpeer_vec(p, rowptr, colind, val, xa, y, fb, st, nnz);
         } else {
-            SpmvBody<false, false, int64_t, XPeer> body{rowptr, colind, val, xa, y};
+            SpmvBody<false, int64_t, XPeer> body{rowptr, colind, val, xa, y};
             body.nnz = nnz;
             s = dispatch(p, body, fb, st);
         }

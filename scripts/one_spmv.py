@@ -20,7 +20,7 @@ ap.add_argument("--hints", type=int, default=0)
 ap.add_argument("--persistent", type=int, default=0)
 ap.add_argument("--iters", type=int, default=3)
 ap.add_argument("--halo", type=int, default=0)
-ap.add_argument("--staged", type=int, default=0)
+ap.add_argument("--tps", type=int, default=0)
 ap.add_argument("--blocked", type=int, default=0)
 ap.add_argument("--vec", type=int, default=0)
 ap.add_argument("--chunk", type=int, default=0)
@@ -39,7 +39,7 @@ for _ in range(a.iters):
     torch.cuda.synchronize()
     P.l2_flush(flush)
     P.spmv_csr_f64(*t, y, simdlen=a.S, mode=a.mode, outer_unroll=a.U, stream_hints=bool(a.hints),
-                   threads_per_team=a.T, persistent=bool(a.persistent), x_halo=a.halo, staged=bool(a.staged), blocked=bool(a.blocked), vec128=a.vec >= 1, quad=a.vec == 2,
+                   threads_per_team=a.T, persistent=bool(a.persistent), x_halo=a.halo, teams_per_sm=a.tps, blocked=bool(a.blocked), vec128=a.vec >= 1, quad=a.vec == 2,
                    team_chunk=a.chunk)
 torch.cuda.synchronize()
 print("done")

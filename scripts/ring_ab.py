@@ -1,0 +1,95 @@
+"""A/B timing of SpMV launch configurations on one matrix (developer tool).
+
+python scripts/ring_ab.py --spec CFG2 [--check]
+Each configuration: median of 10 CUDA-event-timed launches, L2 flushed before
+each.  --check compares every configuration's y with the first one bitwise
+where the lane order is the same, else within R3 against the oracle on a sample.
+"""
+import argparse
+import json
+import os
+import statistics
+import sys
+
+import numpy as np
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import paper_conf_icpp_wrightdtcc23_b200 as P  # noqa: E402
+from nestgen import recipes as R  # noqa: E402
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--spec", default="CFG2")
+ap.add_argument("--iters", type=int, default=10)
+ap.add_argument("--check", action="store_true")
+ap.add_argument("--configs", default="default")
+a = ap.parse_args()
+spec = getattr(R, a.spec)
+rp, col, val = R.spmv_matrix(spec)
+x = R.spmv_x(spec)
+nnz = val.size
+B = nnz * 12 + (spec.nrows + 1) * 8 + spec.nrows * 8 + spec.ncols * 8
+t = [torch.from_numpy(v).cuda() for v in (rp, col, val, x)]
+flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
+
+base = dict(threads_per_team=1024, blocked=True)
+CONFIGS = {
+    "default": [
+        ("nest S2 pairs (r1 headline)", dict(simdlen=2, vec128=True, **base)),
+        ("nest S1 pairs", dict(simdlen=1, vec128=True, **base)),
+        ("ring S2 pairs T768 tps2", dict(simdlen=2, vec128=True, x_halo=4096, teams_per_sm=2, threads_per_team=768)),
+        ("ring S2 pairs T768 tps2 kb2", dict(simdlen=2, vec128=True, x_halo=4096, teams_per_sm=2, outer_unroll=2,
+                                             threads_per_team=768)),
+        ("ring S2 scalar T768 tps2", dict(simdlen=2, x_halo=4096, teams_per_sm=2, threads_per_team=768)),
+        ("ring S2 pairs T1024 tps1", dict(simdlen=2, vec128=True, x_halo=4096, teams_per_sm=1, threads_per_team=1024)),
+        ("ring S4 pairs T768 tps2", dict(simdlen=4, vec128=True, x_halo=4096, teams_per_sm=2, threads_per_team=768)),
+        ("ring S1 pairs T768 tps2", dict(simdlen=1, vec128=True, x_halo=4096, teams_per_sm=2, threads_per_team=768)),
+        ("ring S8 pairs T768 tps2", dict(simdlen=8, vec128=True, x_halo=4096, teams_per_sm=2, threads_per_team=768)),
+        ("ring S2 pairs T768 gsmem", dict(simdlen=2, vec128=True, x_halo=4096, teams_per_sm=2, mode="generic_smem",
+                                          threads_per_team=768)),
+    ],
+}[a.configs]
+
+out = {}
+ys = {}
+for name, cfg in CONFIGS:
+    y = torch.empty(spec.nrows, dtype=torch.float64, device="cuda")
+    try:
+        P.spmv_csr_f64(*t, y, **cfg)
+        torch.cuda.synchronize()
+        plan = P.spmv_plan(spec.nrows, spec.ncols, nnz, **cfg)
+    except P.NestError as e:
+        print(f"{name}: {e}", flush=True)
+        continue
+    ts = []
+    for _ in range(a.iters):
+        P.l2_flush(flush)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        P.spmv_csr_f64(*t, y, **cfg)
+        e1.record()
+        ts.append((e0, e1))
+    torch.cuda.synchronize()
+    ms = statistics.median(a.elapsed_time(b) for a, b in ts)
+    out[name] = {"ms": ms, "GBs": B / ms / 1e6, "plan": plan}
+    ys[name] = y
+    print(f"{name:34s} {ms:.4f} ms  {B / ms / 1e6:7.1f} GB/s  grid {plan['grid']} smem {plan['smem_bytes']} "
+          f"segs {plan['ring_segments']} rowslots {plan['ring_row_slots']}", flush=True)
+
+if a.check:
+    import oracle
+    rng = np.random.default_rng(3)
+    starts = np.concatenate([[0, spec.nrows - 256], rng.integers(0, spec.nrows - 256, 40)])
+    for s in starts:
+        rpl, cl, vl = R.spmv_matrix(spec, row_begin=int(s), nrows=256)
+        yr, ar = oracle.spmv_csr_f64(rpl, cl, vl, x)
+        for name, y in ys.items():
+            yy = y[s:s + 256].cpu().numpy()
+            err = np.abs(yy - yr)
+            assert np.all(err <= 1e-12 * ar), (name, s, float(np.max(err / np.maximum(ar, 1e-300))))
+    # same lane order -> same bits
+    pairs = [k for k in ys if "pairs" in k and "S2" in k]
+    for k in pairs[1:]:
+        assert torch.equal(ys[pairs[0]], ys[k]), (pairs[0], k)
+    print("check ok", flush=True)
+print(json.dumps(out))

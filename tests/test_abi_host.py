@@ -73,15 +73,15 @@ def test_plan_rejects_invalid(cfg):
     assert e.value.status == N.NEST_ERR_INVALID_ARG
 
 
-def test_plan_rejects_bad_abi_version_and_reserved():
+def test_plan_rejects_bad_abi_version_and_teams_per_sm():
     d = P.make_desc()
     d.abi_version = 99
     info = N.nest_plan_info()
     assert N.nest_plan(ctypes.byref(d), 10, 0, ctypes.byref(info)) == N.NEST_ERR_INVALID_ARG
     d = P.make_desc()
-    d.reserved = 5
+    d.teams_per_sm = 1
     assert N.nest_plan(ctypes.byref(d), 10, 0, ctypes.byref(info)) == N.NEST_ERR_INVALID_ARG
-    assert b"reserved" in N.nest_last_error()
+    assert b"teams_per_sm" in N.nest_last_error()
 
 
 def test_invalid_args_rejected_before_any_launch():
@@ -136,3 +136,91 @@ def test_region_program_validates_before_any_device_call():
     assert N.nest_region_program(ctypes.byref(d), regs, 1, None) == N.NEST_ERR_INVALID_ARG
     d.reduce = N.NEST_REDUCE_MAX
     assert N.nest_region_program(ctypes.byref(d), regs, 1, None) == N.NEST_ERR_UNSUPPORTED
+
+
+# ---------------------------------------------------------------- nest_spmv_plan (a1 for a8)
+# Generic payload = sizeof(Slot{int32 fn, int32 count, Loop}) of the body that RUNS
+# (the plan used to report the 64-bit scalar body's 24 bytes for every
+# variant).  Loop: scalar {I trip, I base}; 128-bit tuples {I base, int32 trip, int32 len}.
+SLOT_HEADER = 8
+
+
+def expected_payload(vec, bits):
+    if vec:
+        return SLOT_HEADER + (bits // 8) + 8 if bits == 32 else SLOT_HEADER + 16
+    return SLOT_HEADER + 2 * (bits // 8)
+
+
+@pytest.mark.parametrize("vec", [False, True])
+@pytest.mark.parametrize("S", SIMDLENS)
+@pytest.mark.parametrize("T", [64, 256, 1024])
+@pytest.mark.parametrize("sharing", [0, 256, 2048, 8192])
+def test_spmv_plan_payload_and_fallback_are_the_launched_bodys(vec, S, T, sharing):
+    nrows, ncols = 10_000, 10_000
+    for nnz, bits in ((80_000, 32), ((1 << 31) + 100, 64)):
+        info = P.spmv_plan(nrows, ncols, nnz, simdlen=S, threads_per_team=T, mode="generic_smem",
+                           sharing_bytes=sharing, num_teams=5, vec128=vec)
+        assert info["kernel"] == N.NEST_KERNEL_NEST and info["index_bits"] == bits
+        assert info["payload_bytes"] == expected_payload(vec, bits)
+        G = T // S
+        slot = ((sharing or 2048) // G) & ~7
+        assert info["slot_bytes"] == slot
+        # global fallback exactly when the payload exceeds the slot
+        assert info["uses_global_fallback"] == (int(info["payload_bytes"] > slot) if S > 1 else 0)
+
+
+def test_spmv_plan_fallback_flips_at_the_bodys_own_size():
+    # S = 2, T = 256: G = 128; a 2048-byte space gives 16-byte slots.  The 32-bit
+    # scalar body posts 16 bytes (fits); the 32-bit pair body 20 (global fallback).
+    base = dict(simdlen=2, threads_per_team=256, mode="generic_smem", num_teams=3)
+    assert P.spmv_plan(1000, 1000, 8000, **base)["uses_global_fallback"] == 0
+    assert P.spmv_plan(1000, 1000, 8000, vec128=True, **base)["uses_global_fallback"] == 1
+    # SPMD never uses the sharing space
+    assert P.spmv_plan(1000, 1000, 8000, vec128=True, **dict(base, mode="spmd"))["uses_global_fallback"] == 0
+
+
+@pytest.mark.parametrize("S", SIMDLENS)
+@pytest.mark.parametrize("T,tps", [(64, 0), (256, 0), (768, 2), (1024, 1), (1024, 0)])
+@pytest.mark.parametrize("U", [1, 2, 4])
+def test_spmv_plan_x_ring_geometry(S, T, tps, U):
+    H, nrows = 4096, 1_000_000
+    G = (T - 32) // S                      # the last warp is the copy engine
+    R = G * U
+    span = -(-(R + 2 * H) // 256) + 1      # segments one round's window can touch
+    cfg = dict(simdlen=S, threads_per_team=T, x_halo=H, outer_unroll=U, teams_per_sm=tps, num_teams=17,
+               vec128=True)
+    budget = (228 * 1024) // (tps or 1) - 1024
+    stages = (T // 32 - 1) * 4 * ((U * (32 // S + 1) + 1) & ~1) * 8   # row-bound stages of the consumer warps
+    if (span + 1) * 2064 + stages > budget:   # the forced team count cannot hold one round's window
+        with pytest.raises(P.NestError) as e:
+            P.spmv_plan(nrows, nrows, 8 * nrows, **cfg)
+        assert e.value.status == N.NEST_ERR_UNSUPPORTED
+        return
+    info = P.spmv_plan(nrows, nrows, 8 * nrows, **cfg)
+    assert info["kernel"] == N.NEST_KERNEL_XRING and info["groups_per_team"] == G
+    assert info["ring_segments"] >= span + 1
+    assert info["smem_bytes"] <= 227 * 1024
+    assert info["ring_segments"] * 2048 <= info["smem_bytes"]
+    assert info["grid"] == 17 and info["chunk"] == -(-nrows // 17)
+    assert info["payload_bytes"] == expected_payload(True, 32)
+
+
+def test_spmv_plan_x_ring_rejections():
+    with pytest.raises(P.NestError) as e:    # one warp: no consumer beside the copy warp
+        P.spmv_plan(1000, 1000, 8000, x_halo=100, threads_per_team=32, num_teams=1)
+    assert e.value.status == N.NEST_ERR_INVALID_ARG
+    with pytest.raises(P.NestError) as e:    # the window cannot fit shared memory
+        P.spmv_plan(1000, 1000, 8000, x_halo=200_000, num_teams=1)
+    assert e.value.status == N.NEST_ERR_UNSUPPORTED
+    with pytest.raises(P.NestError) as e:    # quads are not offered with the ring
+        P.spmv_plan(1000, 1000, 8000, x_halo=100, quad=True, num_teams=1)
+    assert e.value.status == N.NEST_ERR_UNSUPPORTED
+    with pytest.raises(P.NestError) as e:    # teams_per_sm only with the ring
+        P.spmv_plan(1000, 1000, 8000, teams_per_sm=2, num_teams=1)
+    assert e.value.status == N.NEST_ERR_INVALID_ARG
+    with pytest.raises(P.NestError) as e:    # two teams per SM need T <= 768 (registers)
+        P.spmv_plan(1000, 1000, 8000, x_halo=100, teams_per_sm=2, threads_per_team=1024, num_teams=1)
+    assert e.value.status == N.NEST_ERR_UNSUPPORTED
+    with pytest.raises(P.NestError) as e:    # the removed staged-pipeline bit is an unknown flag
+        P.spmv_plan(1000, 1000, 8000, flags=1 << 2, num_teams=1)
+    assert e.value.status == N.NEST_ERR_INVALID_ARG

@@ -1,0 +1,120 @@
+"""GPU parity at BASELINE.json's full sizes, EVERY output element against the
+oracle (sampled rows can miss team-chunk and persistent-grid
+tails).  The launch configurations are the ones bench.py times (its headline,
+its simdlen-1 comparison point, the x ring) plus the cfg5 / cfg4 bests.
+Bars as tests/test_gpu_parity.py: R3 (|y - ref| <= 1e-12 * sum|terms| per row,
+fp64; 1e-5 fp32), +0.0 exactly where sum|terms| == 0.
+"""
+import numpy as np
+import pytest
+
+import oracle
+from nestgen import recipes as R
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def P():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_icpp_wrightdtcc23_b200 as P
+    return P
+
+
+def assert_close(y, ref, absref, tol, what=""):
+    y = np.asarray(y, np.float64)
+    zero = absref == 0
+    assert np.all(y[zero] == 0.0) and not np.signbit(y[zero]).any(), f"{what}: abs_ref == 0 must give +0.0"
+    err = np.abs(y - ref)
+    bad = err > tol * absref
+    assert not bad.any(), (f"{what}: {bad.sum()} of {y.size} rows beyond {tol}*abs, first at "
+                           f"{int(np.argmax(bad))}")
+
+
+def bench_configs():
+    import bench
+    return [("headline", bench.cfg_of(bench.HEADLINE))] + [
+        (f"cand{c}", bench.cfg_of(c)) for c in bench.CANDIDATES if c[0] == 1][:2]
+
+
+RING = dict(simdlen=2, mode="spmd", threads_per_team=1024, x_halo=4096, vec128=True)
+
+
+@pytest.mark.parametrize("spec_name", ["CFG2", "G100", "CFG2_UNIFORM"])
+def test_spmv_full_size_every_row(P, spec_name):
+    spec = getattr(R, spec_name)
+    rp, col, val = R.spmv_matrix(spec)
+    x = R.spmv_x(spec)
+    yref, aref = oracle.spmv_csr_f64(rp, col, val, x)
+    t = [torch.from_numpy(a).cuda() for a in (rp, col, val, x)]
+    del rp, col, val
+    y = torch.empty(spec.nrows, dtype=torch.float64, device="cuda")
+    cfgs = bench_configs() + [("ring S2 pairs", RING), ("ring S1 pairs", dict(RING, simdlen=1)),
+                              ("ring S8 scalar generic", dict(RING, simdlen=8, vec128=False, mode="generic_smem")),
+                              ("S8 pairs", dict(simdlen=8, threads_per_team=1024, blocked=True, vec128=True))]
+    for name, cfg in cfgs:
+        y.fill_(np.nan)
+        P.spmv_csr_f64(*t, y, **cfg)
+        assert_close(y.cpu().numpy(), yref, aref, 1e-12, f"{spec_name} {name}")
+    del t, y
+    torch.cuda.empty_cache()
+
+
+def test_spmv_cfg5_full_size_every_row(P):
+    """configs[4] on ONE GPU (100M rows, 1.6G nonzeros, 21.6 GB): generated in row
+    chunks straight into device memory, the oracle run on each chunk as it is
+    generated, then every row of the launch compared."""
+    spec = R.CFG5
+    free, _ = torch.cuda.mem_get_info()
+    if free < 30 << 30:
+        pytest.skip("cfg5 needs ~24 GB of device memory")
+    n = spec.nrows
+    x = R.spmv_x(spec)
+    dx = torch.from_numpy(x).cuda()
+    drp = torch.empty(n + 1, dtype=torch.int64, device="cuda")
+    # nnz first (row lengths only), then the arrays
+    chunk = 10_000_000
+    lens_total = 0
+    bounds = []
+    for r0 in range(0, n, chunk):
+        m = min(chunk, n - r0)
+        rp = R.spmv_matrix(spec, row_begin=r0, nrows=m)[0]
+        bounds.append((r0, m, lens_total))
+        lens_total += int(rp[-1])
+    dcol = torch.empty(lens_total, dtype=torch.int32, device="cuda")
+    dval = torch.empty(lens_total, dtype=torch.float64, device="cuda")
+    yref = np.empty(n)
+    aref = np.empty(n)
+    for r0, m, z0 in bounds:
+        rp, col, val = R.spmv_matrix(spec, row_begin=r0, nrows=m)
+        yref[r0:r0 + m], aref[r0:r0 + m] = oracle.spmv_csr_f64(rp, col, val, x)
+        drp[r0:r0 + m + 1] = torch.from_numpy(rp + z0)
+        dcol[z0:z0 + col.size] = torch.from_numpy(col)
+        dval[z0:z0 + val.size] = torch.from_numpy(val)
+        del rp, col, val
+    y = torch.empty(n, dtype=torch.float64, device="cuda")
+    for name, cfg in (("S8 pairs blocked", dict(simdlen=8, threads_per_team=1024, blocked=True, vec128=True)),
+                      ("ring S8 pairs", dict(RING, simdlen=8)),
+                      ("S1 pairs blocked", dict(simdlen=1, threads_per_team=1024, blocked=True, vec128=True))):
+        y.fill_(np.nan)
+        P.spmv_csr_f64(drp, dcol, dval, dx, y, **cfg)
+        assert_close(y.cpu().numpy(), yref, aref, 1e-12, f"cfg5 {name}")
+    del drp, dcol, dval, dx, y
+    torch.cuda.empty_cache()
+
+
+def test_batched_cfg4_full_size_every_row(P):
+    """configs[3]: 500k batches of 64x64 fp32 -- every y[b][r] against the fp64
+    oracle rounded once (R3 at 1e-5)."""
+    B = 500_000
+    A, x = R.batched_inputs(B)
+    yref, aref = oracle.batched_matvec_f32(A, x, B)
+    dA, dx = torch.from_numpy(A).cuda(), torch.from_numpy(x).cuda()
+    del A
+    for S, mode, vec in ((4, "spmd", True), (1, "spmd", True), (8, "generic_smem", False)):
+        y = P.batched_matvec_f32(dA, dx, B, simdlen=S, mode=mode, vec128=vec, threads_per_team=256)
+        assert_close(y.cpu().numpy(), yref, aref, 1e-5, f"cfg4 S{S} {mode}")
+    del dA, dx
+    torch.cuda.empty_cache()

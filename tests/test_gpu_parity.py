@@ -342,7 +342,7 @@ def test_stencil_max_and_cfg3_full(P):
         assert np.array_equal(host(P.nested_stencil_f64(*t, N, L, simdlen=16, reduce="max")), ymax)
 
 
-# ------------------------------------------------------------------ a8 SpMV, x window
+# ------------------------------------------------------------------ a8 SpMV, x ring
 @pytest.fixture(scope="module")
 def banded():
     out = {}
@@ -354,23 +354,44 @@ def banded():
     return out
 
 
+# (x_halo, rows per group per round, T, num_teams, teams_per_sm, 128-bit pairs)
+RING_CASES = ((700, 1, 256, 0, 0, False), (64, 2, 512, 0, 0, True), (4096, 4, 256, 0, 0, False),
+              (1, 1, 1024, 0, 2, True), (700, 2, 256, 5, 0, False), (3000, 1, 128, 1, 0, True),
+              (4096, 1, 1024, 0, 1, True), (700, 1, 64, 3, 0, False))
+
+
 @pytest.mark.parametrize("S", SIMDLENS)
 @pytest.mark.parametrize("mode", MODES)
-def test_spmv_xwin(P, banded, S, mode):
+def test_spmv_ring(P, banded, S, mode):
+    """x ring (spmv_ring_kernel) against the oracle, and bit-identical to nest_kernel
+    at the same simdlen, mode and loads (same per-lane order, R1/R20)."""
     for values in ("int", "real"):
         rp, col, val, x, yref, aref = banded[values]
         t = [dev(rp), dev(col), dev(val), dev(x)]
-        for halo, U, T, teams in ((700, 1, 256, 0), (64, 2, 512, 0), (4096, 4, 256, 0),
-                                  (1, 1, 1024, 0), (700, 2, 256, 5), (3000, 1, 128, 1)):
-            y = host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, outer_unroll=U, threads_per_team=T,
-                                    x_halo=halo, num_teams=teams))
+        ynest = {vec: host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, vec128=vec)) for vec in (False, True)}
+        for halo, U, T, teams, tps, vec in RING_CASES:
+            cfg = dict(simdlen=S, mode=mode, outer_unroll=U, threads_per_team=T, x_halo=halo, num_teams=teams,
+                       teams_per_sm=tps, vec128=vec)
+            assert P.spmv_plan(rp.size - 1, x.size, val.size, **cfg)["kernel"] == 1
+            y = host(P.spmv_csr_f64(*t, **cfg))
             if values == "int":
-                assert np.array_equal(bits(y), bits(yref)), (halo, U, T, teams)
+                assert np.array_equal(bits(y), bits(yref)), cfg
             else:
                 assert_close(y, yref, aref, 1e-12)
+            assert np.array_equal(bits(y), bits(ynest[vec])), cfg
 
 
-def test_spmv_xwin_cfg1_and_rectangular(P, cfg1):
+@pytest.mark.parametrize("op", ["max", "min"])
+def test_spmv_ring_max_min(P, banded, op):
+    rp, col, val, x, _, _ = banded["real"]
+    yref, _ = oracle.spmv_csr_f64(rp, col, val, x, op=op)
+    t = [dev(rp), dev(col), dev(val), dev(x)]
+    for S, mode, vec in ((1, "spmd", True), (4, "generic_smem", False), (32, "generic_shfl", True)):
+        y = host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, reduce=op, x_halo=700, vec128=vec, threads_per_team=512))
+        assert np.array_equal(y, yref)
+
+
+def test_spmv_ring_cfg1_and_rectangular(P, cfg1):
     rp, col, val, x, yref, aref = cfg1["int"]
     t = [dev(rp), dev(col), dev(val), dev(x)]
     for S in (1, 8, 32):
@@ -378,82 +399,59 @@ def test_spmv_xwin_cfg1_and_rectangular(P, cfg1):
             y = host(P.spmv_csr_f64(*t, simdlen=S, x_halo=halo, mode="generic_smem", sharing_bytes=64))
             assert np.array_equal(bits(y), bits(yref))
     # more rows than columns: windows past the last column are empty
-    rows = [[(c, 1.0) for c in (0, 3)]] * 3000
     rp2 = np.arange(0, 2 * 3000 + 1, 2, dtype=np.int64)
     col2 = np.tile(np.array([0, 3], np.int32), 3000)
     x2 = np.array([1.5, 0, 0, 2.0])
     y = host(P.spmv_csr_f64(dev(rp2), dev(col2), dev(np.ones(6000)), dev(x2), simdlen=2, x_halo=8))
     assert np.all(y == 3.5)
-    del rows
 
 
-def test_spmv_xwin_too_big_is_unsupported(P, cfg1):
-    rp, col, val, x, _, _ = cfg1["int"]
-    with pytest.raises(P.NestError) as e:
-        P.spmv_csr_f64(dev(rp), dev(col), dev(val), dev(x), simdlen=1, threads_per_team=1024,
-                       outer_unroll=4, x_halo=20000)
-    assert e.value.status == 2
-
-
-# ------------------------------------------------------------------ a8 SpMV, staged pipeline
-@pytest.mark.parametrize("S", SIMDLENS)
-@pytest.mark.parametrize("mode", MODES)
-def test_spmv_staged(P, banded, S, mode):
-    for values in ("int", "real"):
-        rp, col, val, x, yref, aref = banded[values]
-        t = [dev(rp), dev(col), dev(val), dev(x)]
-        for halo, U, T, teams in ((0, 1, 256, 0), (700, 1, 1024, 0), (64, 2, 512, 0), (4096, 4, 128, 0),
-                                  (1, 2, 128, 0), (700, 1, 256, 3), (300, 4, 1024, 1)):
-            if (T - 96) // S == 0:
-                continue
-            y = host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, outer_unroll=U, threads_per_team=T,
-                                    x_halo=halo, num_teams=teams, staged=True))
-            if values == "int":
-                assert np.array_equal(bits(y), bits(yref)), (halo, U, T, teams)
-            else:
-                assert_close(y, yref, aref, 1e-12)
-
-
-def test_spmv_staged_long_rows_and_odd_sizes(P):
-    # rows longer than any stage (global path), odd nnz / ncols (unaligned tails)
+def test_spmv_ring_long_rows_and_odd_sizes(P):
+    # rows far longer than a round's share, odd nnz / ncols (the copy engine's hand-copied
+    # tails), empty matrices and empty rows, more teams than rows
     for lens, ncols in (([0, 3, 40000, 7, 1, 0, 25000, 5] * 3 + [1], 60001),
-                        ([1] * 999 + [2], 1001), ([0] * 50, 7)):
+                        ([1] * 999 + [2], 1001), ([0] * 50, 7), ([3] * 5, 257)):
         rp, col, val, x = _rows_matrix(lens, ncols, 11)
         yref, _ = oracle.spmv_csr_f64(rp, col, val, x)
         t = [dev(rp), dev(col), dev(val), dev(x)]
         for S in (1, 4, 32):
             for mode in MODES:
-                for halo in (0, 3, 1000):
-                    y = host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, x_halo=halo, staged=True,
-                                            threads_per_team=256))
-                    assert np.array_equal(bits(y), bits(yref)), (lens[:3], S, mode, halo)
+                for halo, T, teams in ((3, 256, 0), (1000, 128, 0), (300, 1024, 40)):
+                    for vec in (False, True):
+                        y = host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, x_halo=halo, threads_per_team=T,
+                                                num_teams=teams, vec128=vec))
+                        assert np.array_equal(bits(y), bits(yref)), (lens[:3], S, mode, halo, T, vec)
 
 
-def test_spmv_staged_cfg2_full_size_sampled(P):
-    spec = R.CFG2
-    rp, col, val = R.spmv_matrix(spec)
-    x = R.spmv_x(spec)
-    t = [dev(rp), dev(col), dev(val), dev(x)]
-    rng = np.random.default_rng(8)
-    starts = np.concatenate([[0, spec.nrows - 64], rng.integers(0, spec.nrows - 64, 20)])
-    ref = {int(s): oracle.spmv_csr_f64(*R.spmv_matrix(spec, row_begin=int(s), nrows=64), x) for s in starts}
-    for S, mode, U, T, halo in ((8, "spmd", 2, 1024, 4096), (4, "generic_smem", 2, 512, 4096),
-                                (16, "generic_shfl", 1, 1024, 4096), (1, "spmd", 1, 256, 4096),
-                                (8, "spmd", 1, 1024, 0)):
-        y = host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, outer_unroll=U, threads_per_team=T,
-                                x_halo=halo, staged=True))
-        for s, (yr, ar) in ref.items():
-            assert_close(y[s:s + 64], yr, ar, 1e-12)
-
-
-def test_spmv_staged_alignment_and_small_team(P, cfg1):
-    rp, col, val, x, _, _ = cfg1["int"]
-    dcol = torch.from_numpy(np.concatenate([[0], col]).astype(np.int32)).cuda()[1:]
+def test_spmv_ring_misaligned_rowptr_and_x(P, banded):
+    """rowptr at an 8-byte (not 16-byte) offset: the copy engine copies the first
+    entry of such a round by hand (no misaligned bulk copy); an
+    unaligned x is refused before any launch."""
+    rp, col, val, x, yref, _ = banded["int"]
+    big = torch.from_numpy(np.concatenate([[0], rp])).cuda()
+    rp_off = big[1:]
+    assert rp_off.data_ptr() % 16 == 8
+    for S, U, T in ((2, 1, 1024), (4, 2, 256), (1, 1, 128)):
+        y = host(P.spmv_csr_f64(rp_off, dev(col), dev(val), dev(x), simdlen=S, x_halo=700, outer_unroll=U,
+                                threads_per_team=T))
+        assert np.array_equal(bits(y), bits(yref))
+    xb = torch.from_numpy(np.concatenate([[0.0], x])).cuda()[1:]
     with pytest.raises(P.NestError) as e:
-        P.spmv_csr_f64(dev(rp), dcol, dev(val), dev(x), staged=True)
+        P.spmv_csr_f64(dev(rp), dev(col), dev(val), xb, x_halo=700)
     assert e.value.status == 2
+
+
+def test_spmv_ring_too_big_is_unsupported(P, cfg1):
+    rp, col, val, x, _, _ = cfg1["int"]
     with pytest.raises(P.NestError) as e:
-        P.spmv_csr_f64(dev(rp), dev(col), dev(val), dev(x), staged=True, threads_per_team=96)
+        P.spmv_csr_f64(dev(rp), dev(col), dev(val), dev(x), simdlen=1, threads_per_team=1024,
+                       outer_unroll=4, x_halo=20000)
+    assert e.value.status == 2
+    with pytest.raises(P.NestError) as e:   # quads are not offered with the ring
+        P.spmv_csr_f64(dev(rp), dev(col), dev(val), dev(x), x_halo=100, quad=True)
+    assert e.value.status == 2
+    with pytest.raises(P.NestError) as e:   # the copy warp needs a consumer warp beside it
+        P.spmv_csr_f64(dev(rp), dev(col), dev(val), dev(x), x_halo=100, threads_per_team=32)
     assert e.value.status == 1
 
 

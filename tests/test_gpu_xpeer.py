@@ -92,8 +92,8 @@ def test_xpeer_odd_chunks_and_errors(P):
         assert np.array_equal(bits(y), bits(y1[rb:rb + nloc]))
         with pytest.raises(P.NestError):          # wrong local row count
             xp.spmv_csr_f64(spec.nrows + 50, *t)
-        with pytest.raises(P.NestError):          # staged variant is not offered here
-            xp.spmv_csr_f64(spec.nrows, *t, staged=True, threads_per_team=256)
+        with pytest.raises(P.NestError):          # the x ring is not offered here
+            xp.spmv_csr_f64(spec.nrows, *t, x_halo=100, threads_per_team=256)
         xp.close()
 
 
