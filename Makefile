@@ -24,9 +24,10 @@ host: nestgen/libnestgen.so oracle/liboracle.so
 nestgen/libnestgen.so: nestgen/nestgen.c
 	$(CC) -O2 -fopenmp -fPIC -shared -o $@ $<
 
-# The oracle: plain C, no FMA contraction, no fast-math, single-threaded.
+# The oracle: plain C, no FMA contraction, no fast-math; single-threaded except
+# oracle_spmv_csr_f64_threads (OpenMP over rows, the all-cores CPU baseline).
 oracle/liboracle.so: oracle/oracle.c
-	$(CC) -O2 -ffp-contract=off -fno-fast-math -fPIC -shared -o $@ $< -lm
+	$(CC) -O2 -ffp-contract=off -fno-fast-math -fopenmp -fPIC -shared -o $@ $< -lm
 
 build/%.o: $(CSRC)/%.cu $(CU_HDRS)
 	@mkdir -p build

@@ -1,17 +1,26 @@
 """Benchmark: the three-level CSR SpMV hot path on B200 (BASELINE.json metric
 "3-level SpMV GB/s vs HBM peak; speedup over simd-folded 2-level mapping").
 
-One step = one y = A x over BASELINE.json configs[1] (10M x 10M CSR, nnz/row
-U{4..12} banded+far, fp64) through the C ABI, in the best (simdlen, mode,
-variant) found by a short untimed autotune; the simd-folded two-level mapping
-(simdlen = 1) is timed the same way for the speedup.
-
   python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
 
-N > 1 (torchrun, one rank per GPU): the row-partitioned SpMV with the NCCL
-all-gather of x (BASELINE.json configs[4] scheme), weak scaling with 10M rows
-per rank.  --impl reference times the CPU oracle (the only reference this
-paper-only tier has) on the same workload.  Prints ONE JSON line on rank 0.
+N = 1: one step = one y = A x over BASELINE.json configs[1] (10M x 10M CSR,
+nnz/row U{4..12} banded+far, fp64) through the C ABI in the headline
+configuration (simdlen 2, SPMD, blocked teams, 128-bit pairs); ``value`` is its
+algorithmic GB/s.  The same line carries the simd-folded two-level mapping
+(simdlen 1) timed the same way, a short sweep of (simdlen, mode, variant), the
+north_star's 100M-nnz gate matrix (G100) and configs[4] on one GPU (100M rows,
+1.6G nonzeros) as extra legs with their own roofline, the end-to-end call from
+pinned host buffers, and the CPU oracle (1 thread and all cores).
+
+N > 1 (torchrun, one rank per GPU): configs[4] -- 100M rows, U{8..24} nnz/row --
+row-partitioned over the ranks at FIXED total size (strong scaling); each rank
+generates only its own rows.  A step is the NCCL all-gather of x plus the local
+SpMV (a12); the all-gather and the local SpMV are also timed alone, the peer-
+gather variant (NEXT-4) beside them, every rank's rows are checked against the
+oracle, and the line carries the end-to-end host-buffer call.
+
+--impl reference: the CPU oracle (this paper-only tier has no installable
+reference implementation) on the same workload, rank 0 only.
 """
 from __future__ import annotations
 
@@ -33,12 +42,20 @@ from nestgen import recipes as R  # noqa: E402
 METRIC = "3-level SpMV GB/s vs HBM peak; speedup over simd-folded 2-level mapping"
 UNIT = "GB/s"
 SPEC = R.CFG2
+SPEC_MULTI = R.CFG5
+FLUSH_BYTES = 512 << 20   # 4x the 126 MB L2
 
 
 def alg_bytes(nrows: int, ncols: int, nnz: int) -> int:
     """Algorithmic bytes of one SpMV: the CSR arrays once,
     x once, y written once."""
     return nnz * (8 + 4) + (nrows + 1) * 8 + nrows * 8 + ncols * 8
+
+
+def workload(spec, which: str = "configs[1]") -> str:
+    """The workload string -- identical in both arms (--impl ours / reference)."""
+    return (f"{spec.name}: CSR SpMV fp64 {spec.nrows}x{spec.ncols}, nnz/row U{{{spec.nnz_min}..{spec.nnz_max}}} "
+            f"banded+far (W={spec.band_w}, far 1/{spec.far_den}), seed {spec.seed} (BASELINE.json {which})")
 
 
 def peaks():
@@ -48,6 +65,16 @@ def peaks():
         return float(p["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
     except Exception:
         return 6650.0, "fallback (B200_PROFILING.md)"
+
+
+def traffic_of(key: str):
+    """ncu dram read+write bytes per launch for a (workload, config) key, from the
+    committed capture summary profiles/traffic.json (None if not captured)."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
+            return json.load(f).get(key)
+    except Exception:
+        return None
 
 
 class ClockSampler:
@@ -104,26 +131,6 @@ class ClockSampler:
                 "reasons": sorted(self.reasons)}
 
 
-# ---------------------------------------------------------------- CPU oracle
-def cpu_baseline(spec, min_seconds=10.0, max_seconds=30.0):
-    """The oracle as it stands (plain sequential C, 1 thread) on a bounded
-    sample: whole passes of the same matrix until >= min_seconds."""
-    import oracle
-    rp, col, val = R.spmv_matrix(spec)
-    x = R.spmv_x(spec)
-    B = alg_bytes(spec.nrows, spec.ncols, val.size)
-    passes, t_total = 0, 0.0
-    while t_total < min_seconds and (passes == 0 or t_total + t_total / passes < max_seconds):
-        t0 = time.perf_counter()
-        oracle.spmv_csr_f64(rp, col, val, x)
-        t_total += time.perf_counter() - t0
-        passes += 1
-    return {"value": B * passes / t_total / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
-            "sample": f"{passes} full passes of {spec.name} ({spec.nrows} rows, {val.size} nnz), "
-                      f"{t_total:.1f} s single-threaded C (oracle/oracle.c)",
-            "host": host_cpu()}
-
-
 def host_cpu():
     """The box's CPU model and logical core count (context for cpu_baseline)."""
     model = "unknown"
@@ -138,15 +145,54 @@ def host_cpu():
     return {"model": model, "logical_cores": os.cpu_count()}
 
 
+# ---------------------------------------------------------------- CPU oracle
+def cpu_baseline(spec, rp, col, val, x, min_seconds=8.0, max_seconds=20.0):
+    """The oracle as it stands on a bounded sample: whole passes of the same
+    matrix for >= min_seconds on ONE thread (the baseline of record), then the
+    same per-row loop on all host cores (OpenMP over rows, bit-identical)."""
+    import oracle
+    B = alg_bytes(spec.nrows, spec.ncols, val.size)
+
+    def timed(fn):
+        passes, t_total = 0, 0.0
+        while t_total < min_seconds and (passes == 0 or t_total + t_total / passes < max_seconds):
+            t0 = time.perf_counter()
+            fn()
+            t_total += time.perf_counter() - t0
+            passes += 1
+        return passes, t_total
+
+    p1, t1 = timed(lambda: oracle.spmv_csr_f64(rp, col, val, x))
+    ncores = os.cpu_count() or 1
+    used = [1]
+
+    def allcores():
+        used[0] = oracle.spmv_csr_f64_threads(rp, col, val, x, ncores)[2]
+    pn, tn = timed(allcores)
+    return {"value": B * p1 / t1 / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"{p1} full passes of {spec.name} ({spec.nrows} rows, {val.size} nnz), {t1:.1f} s, "
+                      "single-threaded C (oracle/oracle.c)",
+            "all_cores": {"value": B * pn / tn / 1e9, "unit": UNIT, "cores": used[0], "kind": "oracle",
+                          "sample": f"{pn} full passes, {tn:.1f} s, the same per-row loop on {used[0]} threads "
+                                    "(OpenMP over rows, bit-identical to 1 thread)"},
+            "host": host_cpu()}
+
+
 def run_reference(args, rank, world):
-    """--impl reference: the oracle on the box's host cores, rank 0 only."""
+    """--impl reference: the oracle on the box's host cores, rank 0 only; the
+    workload string, metric and unit are the GPU arm's.  N = 1: the whole
+    configs[1] matrix per step; N > 1: configs[4] (the GPU arm's workload there)
+    on a bounded sample per step (its first 5M rows), so the run stays short."""
     if rank != 0:
         return
     import oracle
-    spec = SPEC
-    rp, col, val = R.spmv_matrix(spec)
+    if world == 1:
+        spec, which, nrows = SPEC, "configs[1]", SPEC.nrows
+    else:
+        spec, which, nrows = SPEC_MULTI, "configs[4], row-partitioned at fixed total size", 5_000_000
+    rp, col, val = R.spmv_matrix(spec, row_begin=0, nrows=nrows)
     x = R.spmv_x(spec)
-    B = alg_bytes(spec.nrows, spec.ncols, val.size)
+    B = alg_bytes(nrows, spec.ncols, val.size)
     for _ in range(args.warmup):
         oracle.spmv_csr_f64(rp, col, val, x)
     ts = []
@@ -156,60 +202,74 @@ def run_reference(args, rank, world):
         ts.append(time.perf_counter() - t0)
     ms = 1e3 * sum(ts) / len(ts)
     value = B / (ms / 1e3) / 1e9
+    sample = (f"the full {spec.name} matrix per step" if nrows == spec.nrows else
+              f"rows [0, {nrows}) of {spec.name} ({val.size} nnz) per step")
     line = {"metric": METRIC, "value": value, "unit": UNIT, "impl": "reference", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": f"{spec.name}: CSR SpMV fp64 {spec.nrows}x{spec.ncols}, nnz/row "
-                                   f"U{{{spec.nnz_min}..{spec.nnz_max}}} banded+far (W={spec.band_w}, "
-                                   f"far 1/{spec.far_den})", "nnz": int(val.size), "alg_bytes": B},
+            "scaling": "weak" if world == 1 else "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": workload(spec, which), "nnz_per_step": int(val.size), "alg_bytes_per_step": B},
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
-                             "sample": f"the full {spec.name} matrix per step, single-threaded C oracle", "host": host_cpu()},
+                             "sample": f"{sample}, single-threaded C oracle", "host": host_cpu()},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
 
 # ---------------------------------------------------------------- GPU arm
 # (simdlen, mode, outer_unroll, threads_per_team, x_halo, flags) -- flags: "b" blocked
-# team schedule, "s" staged pipeline, "h" streaming cache hints, "v" 128-bit pair
-# loads, "q" 128-bit quad loads
+# team schedule, "v" 128-bit pair loads, "q" 128-bit quad loads, "h" streaming cache
+# hints; x_halo > 0 is the x ring (teams_per_sm chosen by the planner)
 CANDIDATES = [
     (1, "spmd", 1, 256, 0, ""),
-    (1, "spmd", 1, 1024, 0, "b"),
     (1, "spmd", 1, 1024, 0, "bv"),
     (1, "spmd", 1, 1024, 0, "bq"),
     (2, "spmd", 1, 1024, 0, "b"),
     (2, "spmd", 1, 1024, 0, "bv"),
+    (2, "spmd", 1, 1024, 0, "bq"),
     (2, "generic_smem", 1, 1024, 0, "b"),
     (2, "generic_shfl", 1, 1024, 0, "b"),
-    (2, "generic_smem", 1, 1024, 0, "bq"),
-    (4, "spmd", 1, 1024, 0, "b"),
     (4, "spmd", 1, 1024, 0, "bv"),
-    (2, "spmd", 1, 1024, 0, "bq"),
     (4, "spmd", 1, 1024, 0, "bq"),
     (4, "generic_smem", 1, 1024, 0, "b"),
-    (4, "generic_shfl", 1, 1024, 0, "b"),
-    (8, "spmd", 1, 1024, 0, "b"),
+    (8, "spmd", 1, 1024, 0, "bv"),
     (8, "generic_smem", 1, 1024, 0, "b"),
     (16, "spmd", 1, 1024, 0, "b"),
     (32, "spmd", 1, 1024, 0, "b"),
-    (4, "spmd", 1, 512, 4096, "s"),
+    (2, "spmd", 2, 768, 4096, "v"),
 ]
 
 # The headline: the best measured THREE-level configuration (simdlen >= 2; the
 # metric is the 3-level mapping's GB/s): simdlen 2, SPMD, blocked teams of 1024,
 # 128-bit pair loads.  The 2-level comparison point is the best simdlen-1 candidate.
 HEADLINE = (2, "spmd", 1, 1024, 0, "bv")
+SIMDLEN1 = [c for c in CANDIDATES if c[0] == 1]
+# configs[4] (16 nnz/row): wider groups pay (DESIGN.md Fig 9 analogue / cfg5 table)
+HEADLINE_CFG5 = (8, "spmd", 1, 1024, 0, "bv")
 
 
 def cfg_of(c):
     S, mode, U, T, halo, fl = c
     return dict(simdlen=S, mode=mode, outer_unroll=U, threads_per_team=T, x_halo=halo,
-                stream_hints="h" in fl, staged="s" in fl, blocked="b" in fl, vec128="v" in fl or "q" in fl,
-                quad="q" in fl)
+                stream_hints="h" in fl, blocked="b" in fl, vec128="v" in fl or "q" in fl, quad="q" in fl)
 
 
-def time_steps(torch, fn, flush, P, iters, events_out=None):
-    """Per-step CUDA-event times (ms) on the current stream, L2 flushed between steps."""
+def cfg_key(spec, c) -> str:
+    return f"{spec.name}:{json.dumps(list(c))}"
+
+
+def kernel_name(c) -> str:
+    S, mode, U, T, halo, fl = c
+    if halo:
+        return f"spmv_ring_kernel<S={S},{mode},SUM,SpmvVecBody<0,2,int,XRing>>" if "v" in fl else \
+            f"spmv_ring_kernel<S={S},{mode},SUM,SpmvBody<0,int,XRing>>"
+    body = ("SpmvVecBody<0,4,int>" if "q" in fl else "SpmvVecBody<0,2,int>" if "v" in fl
+            else f"SpmvBody<{int('h' in fl)},int>")
+    two_pm = ("v" in fl or "q" in fl) and U == 1 and not ("q" in fl and S == 1)
+    return f"{'nest_kernel_2pm' if two_pm else 'nest_kernel'}<S={S},{mode},SUM,U={U},{body}>"
+
+
+def time_steps(torch, fn, flush, P, iters):
+    """Per-step CUDA-event times (ms) on the current stream (the launching
+    stream), L2 flushed (and left clean) before every step, outside the events."""
     ts = []
     for _ in range(iters):
         P.l2_flush(flush)
@@ -222,7 +282,197 @@ def time_steps(torch, fn, flush, P, iters, events_out=None):
     return [a.elapsed_time(b) for a, b in ts]
 
 
-def run_gpu(args, rank, world, local_rank):
+def roofline(B, ms, peak, peak_src, c, spec):
+    achieved = B / (ms / 1e3) / 1e9
+    traffic = traffic_of(cfg_key(spec, c))
+    return {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+            "traffic": traffic, "peak_source": peak_src,
+            "traffic_source": "profiles/traffic.json: ncu --set full dram__bytes_read.sum + dram__bytes_write.sum "
+                              "per launch (cold L2)",
+            "traffic_over_alg_bytes": (traffic / B) if traffic else None,
+            "alg_bytes_per_launch": B,
+            "alg_bytes_rule": "12 B per nonzero + 16 B per row (rowptr, y) + 8 B per column (x once)",
+            "kernel": kernel_name(c), "frac_of_8TBs_spec": achieved / 8000.0}
+
+
+def gen_to_device(torch, spec, dev, row_begin=0, nrows=None, chunk=10_000_000, with_oracle=False, x=None,
+                  threads=None):
+    """The CSR rows [row_begin, row_begin + nrows) of spec straight into device
+    memory, generated in row chunks (bounded host memory); rowptr is 0-based for
+    the block.  with_oracle: also the oracle's (y, abs) of every row (x given),
+    computed chunk by chunk as it is generated (threaded oracle, bit-identical)."""
+    import oracle
+    n = spec.nrows - row_begin if nrows is None else nrows
+    bounds, total = [], 0
+    for r0 in range(0, n, chunk):
+        m = min(chunk, n - r0)
+        rp = R.spmv_matrix(spec, row_begin=row_begin + r0, nrows=m)[0]   # row lengths only
+        bounds.append((r0, m, total))
+        total += int(rp[-1])
+    drp = torch.empty(n + 1, dtype=torch.int64, device=dev)
+    dcol = torch.empty(total, dtype=torch.int32, device=dev)
+    dval = torch.empty(total, dtype=torch.float64, device=dev)
+    yref = np.empty(n) if with_oracle else None
+    aref = np.empty(n) if with_oracle else None
+    for r0, m, z0 in bounds:
+        rp, col, val = R.spmv_matrix(spec, row_begin=row_begin + r0, nrows=m)
+        if with_oracle:
+            yref[r0:r0 + m], aref[r0:r0 + m], _ = oracle.spmv_csr_f64_threads(rp, col, val, x, threads or
+                                                                              (os.cpu_count() or 1))
+        drp[r0:r0 + m + 1] = torch.from_numpy(rp + z0)
+        dcol[z0:z0 + col.size] = torch.from_numpy(col)
+        dval[z0:z0 + val.size] = torch.from_numpy(val)
+    return drp, dcol, dval, total, yref, aref
+
+
+def parity(y, yref, aref):
+    """R3 on every row: |y - ref| <= 1e-12 * sum|terms|, +0.0 where sum|terms| == 0."""
+    y = np.asarray(y, np.float64)
+    zero = aref == 0
+    err = np.abs(y - yref)
+    rel = np.where(zero, np.where((y == 0) & ~np.signbit(y), 0.0, np.inf), err / np.where(zero, 1.0, aref))
+    worst = float(rel.max()) if rel.size else 0.0
+    return {"rows_checked": int(y.size), "rows_total": int(y.size), "tol": 1e-12, "worst_rel_to_abs": worst,
+            "ok": bool(worst <= 1e-12)}
+
+
+def time_leg(torch, P, spec, c, t, y, flush, iters):
+    fn = lambda: P.spmv_csr_f64(*t, y, **cfg_of(c))
+    fn()
+    ts = time_steps(torch, fn, flush, P, iters)
+    return sum(ts) / len(ts)
+
+
+def run_gpu_single(args, local_rank):
+    import torch
+
+    import oracle
+    import paper_conf_icpp_wrightdtcc23_b200 as P
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    spec = SPEC
+    peak, peak_src = peaks()
+    flush = torch.empty(FLUSH_BYTES, dtype=torch.uint8, device=dev)
+    rp, col, val = R.spmv_matrix(spec)
+    x = R.spmv_x(spec)
+    nnz = int(val.size)
+    pin = lambda a: torch.from_numpy(a).pin_memory()
+    h_rp, h_col, h_val, h_x = pin(rp), pin(col), pin(val), pin(x)
+    t = [h_rp.to(dev), h_col.to(dev), h_val.to(dev), h_x.to(dev)]
+    d_y = torch.empty(spec.nrows, dtype=torch.float64, device=dev)
+    B = alg_bytes(spec.nrows, spec.ncols, nnz)
+
+    # untimed sweep over the candidate (simdlen, mode, variant) set
+    sweep = []
+    for c in CANDIDATES:
+        try:
+            ms_c = time_leg(torch, P, spec, c, t, d_y, flush, 5)
+        except P.NestError as e:
+            print(f"skip {c}: {e}", file=sys.stderr)
+            continue
+        sweep.append((ms_c, c))
+    sweep.sort(key=lambda q: q[0])
+    best = min((q for q in sweep if q[1][0] >= 2), key=lambda q: q[0])[1] if args.autotune else HEADLINE
+    s1 = min((q for q in sweep if q[1][0] == 1), key=lambda q: q[0])[1]
+    cfg = cfg_of(best)
+    step = lambda: P.spmv_csr_f64(*t, d_y, **cfg)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    # timed region: K steps, L2 flushed between steps (flush outside the events)
+    with ClockSampler(local_rank) as clk:
+        torch.cuda.synchronize()
+        ts = time_steps(torch, step, flush, P, args.steps)
+        torch.cuda.synchronize()
+    ms = sum(ts) / len(ts)
+    value = B / (ms / 1e3) / 1e9
+    # parity of the timed configuration: every row against the oracle
+    yref, aref = oracle.spmv_csr_f64(rp, col, val, x)
+    par = parity(d_y.cpu().numpy(), yref, aref)
+    y_head = d_y.clone()
+    # simd-folded two-level mapping (simdlen = 1), same protocol
+    ms1 = time_leg(torch, P, spec, s1, t, d_y, flush, max(5, args.steps // 2))
+
+    # e2e through the C ABI with HOST buffers: H2D of A and x, the SpMV, D2H of y
+    h_y = torch.empty(spec.nrows, dtype=torch.float64).pin_memory()
+    ws = torch.empty(P.hostio_workspace_bytes(spec.nrows, spec.ncols, nnz), dtype=torch.uint8, device=dev)
+    e2e_step = lambda: P.spmv_csr_f64_hostio(h_rp, h_col, h_val, h_x, h_y, ws, **cfg)
+    e2e_step()
+    torch.cuda.synchronize()
+    te = []
+    for _ in range(max(3, min(args.steps, 10))):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        e2e_step()
+        e1.record()
+        e1.synchronize()
+        te.append(e0.elapsed_time(e1))
+    ms_e2e = sum(te) / len(te)
+    e2e_ok = bool(np.array_equal(h_y.numpy().view(np.int64), y_head.cpu().numpy().view(np.int64)))
+    h2d = (spec.nrows + 1) * 8 + nnz * 12 + spec.ncols * 8
+    d2h = spec.nrows * 8
+    cpu = None if args.no_cpu_baseline else cpu_baseline(spec, rp, col, val, x)
+    del t, ws, h_rp, h_col, h_val, h_x, h_y, rp, col, val, y_head
+    torch.cuda.empty_cache()
+
+    # ---- extra legs: the 100M-nnz gate matrix and configs[4] on one GPU
+    legs = {}
+    for lspec, heads, which in ((R.G100, [best, s1], "north_star 70% gate, SURVEY.md §8(d) G100"),
+                                (R.CFG5, [HEADLINE_CFG5, s1], "configs[4] on one GPU")):
+        lx = R.spmv_x(lspec)
+        drp, dcol, dval, lnnz, lyref, laref = gen_to_device(torch, lspec, dev, with_oracle=True, x=lx)
+        lt = [drp, dcol, dval, torch.from_numpy(lx).to(dev)]
+        ly = torch.empty(lspec.nrows, dtype=torch.float64, device=dev)
+        LB = alg_bytes(lspec.nrows, lspec.ncols, lnnz)
+        leg = {"workload": workload(lspec, which), "nnz": lnnz, "alg_bytes": LB, "configs": {}}
+        for c in heads:
+            lms = time_leg(torch, P, lspec, c, lt, ly, flush, 10)
+            leg["configs"][json.dumps(list(c))] = {"ms": lms, "GBs": LB / (lms / 1e3) / 1e9,
+                                                   "roofline": roofline(LB, lms, peak, peak_src, c, lspec),
+                                                   "parity": parity(ly.cpu().numpy(), lyref, laref)}
+        h3 = leg["configs"][json.dumps(list(heads[0]))]
+        leg["headline"] = heads[0]
+        leg["speedup_vs_simdlen1"] = leg["configs"][json.dumps(list(s1))]["ms"] / h3["ms"]
+        legs[lspec.name] = leg
+        del lt, drp, dcol, dval, ly
+        torch.cuda.empty_cache()
+
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": 1, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": workload(spec), "nnz": nnz, "alg_bytes": B, "simdlen": best[0], "mode": best[1],
+                   "outer_unroll": best[2], "threads_per_team": best[3], "x_halo": best[4],
+                   "variant": " + ".join({"b": "blocked teams", "h": "stream hints", "v": "128-bit pair loads",
+                                          "q": "128-bit quad loads"}[f] for f in best[5]) or "cyclic teams",
+                   "l2": "flushed between timed steps (512 MiB write, then a 256 MiB read so L2 holds only clean "
+                         "lines)",
+                   "parallelism": "1 GPU"},
+        "parity": par,
+        "speedup_vs_simdlen1": ms1 / ms,
+        "simdlen1": {"ms_per_step": ms1, "GBs": B / (ms1 / 1e3) / 1e9, "config": cfg_of(s1)},
+        "sweep_ms": {json.dumps(list(c)): round(m, 4) for m, c in sweep},
+        "roofline": roofline(B, ms, peak, peak_src, best, spec),
+        "legs": legs,
+        "e2e": {"value": B / (ms_e2e / 1e3) / 1e9, "unit": UNIT, "h2d_bytes_per_step": h2d,
+                "d2h_bytes_per_step": d2h, "ms_per_step": ms_e2e, "h2d_gbs": h2d / (ms_e2e / 1e3) / 1e9,
+                "bitwise_equal_device_call": e2e_ok,
+                "pipeline": f"{min(32, max(1, -(-nnz // (8 << 20))))} row chunks of ~8 Mi nonzeros: chunk c's "
+                            "SpMV and y copy overlap the H2D of chunks > c (nest_spmv_csr_f64_hostio)"},
+        "gpu_launches": 3 * args.steps,
+        "gpu_launches_detail": "per step: 1 SpMV kernel + 2 l2 flush kernels (write, clean-read; outside the "
+                               "step events)",
+        "clocks": clk.summary(),
+    }
+    if cpu is not None:
+        line["cpu_baseline"] = cpu
+    print(json.dumps(line), flush=True)
+
+
+def run_gpu_multi(args, rank, world, local_rank):
+    """configs[4] row-partitioned over the ranks at fixed total size."""
     import torch
     import torch.distributed as dist
 
@@ -230,150 +480,30 @@ def run_gpu(args, rank, world, local_rank):
 
     torch.cuda.set_device(local_rank)
     dev = torch.device("cuda", local_rank)
-    spec = SPEC
-    if world > 1:
-        gspec = R.SpmvSpec(f"{spec.name}x{world}", spec.seed, spec.nrows * world, spec.ncols * world,
-                           spec.nnz_min, spec.nnz_max, spec.structure, spec.band_w, spec.far_den)
-        chunk, rb, nloc = P.shard_rows(gspec.nrows, world, rank)
-    else:
-        gspec, rb, nloc = spec, 0, spec.nrows
-    rp, col, val = R.spmv_matrix(gspec, row_begin=rb, nrows=nloc)
-    nnz = int(val.size)
-    pin = lambda a: torch.from_numpy(a).pin_memory()
-    h_rp, h_col, h_val = pin(rp), pin(col), pin(val)
-    d_rp, d_col, d_val = (h_rp.to(dev), h_col.to(dev), h_val.to(dev))
-    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)   # 4x the 126 MB L2
+    spec = SPEC_MULTI
     peak, peak_src = peaks()
-
-    if world == 1:
-        x = R.spmv_x(spec)
-        h_x = pin(x)
-        d_x = h_x.to(dev)
-        d_y = torch.empty(spec.nrows, dtype=torch.float64, device=dev)
-        B = alg_bytes(spec.nrows, spec.ncols, nnz)
-
-        # untimed autotune over the candidate (simdlen, mode, variant) set
-        sweep = []
-        for c in CANDIDATES:
-            cfg = cfg_of(c)
-            fn = lambda cfg=cfg: P.spmv_csr_f64(d_rp, d_col, d_val, d_x, d_y, **cfg)
-            try:
-                fn()
-            except P.NestError as e:
-                print(f"skip {c}: {e}", file=sys.stderr)
-                continue
-            ts = time_steps(torch, fn, flush, P, 5)
-            sweep.append((statistics.median(ts), c))
-        sweep.sort(key=lambda t: t[0])
-        # the timed configuration is fixed (reproducible under a profiler); --autotune
-        # times the fastest candidate of this run's sweep instead
-        best = min((t for t in sweep if t[1][0] >= 2), key=lambda t: t[0])[1] if args.autotune else HEADLINE
-        s1 = min((t for t in sweep if t[1][0] == 1), key=lambda t: t[0])   # best 2-level (simdlen 1)
-        cfg = cfg_of(best)
-        step = lambda: P.spmv_csr_f64(d_rp, d_col, d_val, d_x, d_y, **cfg)
-
-        for _ in range(args.warmup):
-            step()
-        torch.cuda.synchronize()
-        # timed region: K steps, L2 flushed between steps (flush outside the events)
-        with ClockSampler(local_rank) as clk:
-            torch.cuda.synchronize()
-            ts = time_steps(torch, step, flush, P, args.steps)
-            torch.cuda.synchronize()
-        ms = sum(ts) / len(ts)
-        value = B / (ms / 1e3) / 1e9
-        # simd-folded two-level mapping (simdlen = 1), same protocol
-        s1_cfg = cfg_of(s1[1])
-        ts1 = time_steps(torch, lambda: P.spmv_csr_f64(d_rp, d_col, d_val, d_x, d_y, **s1_cfg), flush, P,
-                         max(3, args.steps // 2))
-        ms1 = sum(ts1) / len(ts1)
-
-        # e2e through the C ABI with HOST buffers: H2D of A and x, the SpMV, D2H of y
-        h_y = torch.empty(spec.nrows, dtype=torch.float64).pin_memory()
-        ws = torch.empty(P.hostio_workspace_bytes(spec.nrows, spec.ncols, nnz), dtype=torch.uint8, device=dev)
-        e2e_step = lambda: P.spmv_csr_f64_hostio(h_rp, h_col, h_val, h_x, h_y, ws, **cfg)
-        e2e_step()
-        torch.cuda.synchronize()
-        n_e2e = max(3, min(args.steps, 10))
-        te = []
-        for _ in range(n_e2e):
-            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            e0.record()
-            e2e_step()
-            e1.record()
-            e1.synchronize()
-            te.append(e0.elapsed_time(e1))
-        ms_e2e = sum(te) / len(te)
-        h2d = (spec.nrows + 1) * 8 + nnz * 12 + spec.ncols * 8
-        d2h = spec.nrows * 8
-
-        body = ("SpmvVecBody<0,4>" if "q" in best[5] else "SpmvVecBody<0,2>" if "v" in best[5]
-                else f"SpmvBody<{int('h' in best[5])},0>")
-        kname = ("nest_kernel_2pm" if ("v" in best[5] or "q" in best[5]) and best[2] == 1
-                 and not ("q" in best[5] and best[0] == 1) else "nest_kernel")
-        kernel_name = (f"spmv_staged_kernel<S={best[0]},{best[1]},SUM,U={best[2]}>" if "s" in best[5] else
-                       f"{kname}<S={best[0]},{best[1]},SUM,U={best[2]},{body}>")
-        traffic = None
-        try:
-            with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
-                traffic = json.load(f).get(json.dumps(list(best)))
-
-        except Exception:
-            pass
-        line = {
-            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": 1, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
-            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": f"{spec.name}: CSR SpMV fp64 {spec.nrows}x{spec.ncols}, nnz/row "
-                                   f"U{{{spec.nnz_min}..{spec.nnz_max}}} banded+far (W={spec.band_w}, far "
-                                   f"1/{spec.far_den}), seed {spec.seed} (BASELINE.json configs[1])",
-                       "nnz": nnz, "alg_bytes": B, "simdlen": best[0], "mode": best[1],
-                       "outer_unroll": best[2], "threads_per_team": best[3], "x_halo": best[4],
-                       "variant": " + ".join({"b": "blocked teams", "s": "staged pipeline", "h": "stream hints",
-                                              "v": "128-bit pair loads", "q": "128-bit quad loads"}[f]
-                                             for f in best[5]) or "cyclic teams",
-                       "l2": "flushed between timed steps (512 MiB write, then a 256 MiB read so L2 holds only clean lines)",
-                       "parallelism": "1 GPU"},
-            "speedup_vs_simdlen1": ms1 / ms,
-            "simdlen1": {"ms_per_step": ms1, "GBs": B / (ms1 / 1e3) / 1e9, "config": cfg_of(s1[1])},
-            "sweep_ms": {json.dumps(list(c)): round(t, 4) for t, c in sweep},
-            "roofline": {"bound": "hbm", "achieved": value, "peak": peak, "unit": "GB/s",
-                         "frac": value / peak, "traffic": traffic, "peak_source": peak_src,
-                         "traffic_source": "profiles/traffic.json: dram read+write bytes per launch, ncu --set full",
-                         "traffic_over_alg_bytes": (traffic / B) if traffic else None,
-                         "kernel": kernel_name, "frac_of_8TBs_spec": value / 8000.0},
-            "e2e": {"value": B / (ms_e2e / 1e3) / 1e9, "unit": UNIT, "h2d_bytes_per_step": h2d,
-                    "d2h_bytes_per_step": d2h, "ms_per_step": ms_e2e,
-                    "h2d_gbs": h2d / (ms_e2e / 1e3) / 1e9,
-                    "pipeline": (f"{int(os.environ['NEST_HOSTIO_CHUNKS'])} row chunks (forced)"
-                                 if os.environ.get("NEST_HOSTIO_CHUNKS") else
-                                 f"{min(32, max(1, -(-nnz // (8 << 20))))} row chunks of ~8 Mi nonzeros")
-                    + ": chunk c's SpMV and y copy overlap the H2D of chunks > c"},
-            "gpu_launches": 3 * args.steps,
-            "gpu_launches_detail": "per step: 1 SpMV kernel + 2 l2 flush kernels (write, clean-read; outside the step events)",
-            "clocks": clk.summary(),
-        }
-        if not args.no_cpu_baseline:
-            line["cpu_baseline"] = cpu_baseline(spec)
-        print(json.dumps(line), flush=True)
-        return
-
-    # ---- N > 1: row-partitioned SpMV (weak scaling: spec.nrows rows per rank).
-    # Two exchange strategies, both timed: "xpeer" (NEXT-4, the headline) -- x
-    # stays distributed and the SpMV's simd lanes gather remote x from the
-    # owner's slice over NVLink, bracketed by peer-memory barriers -- and
-    # "allgather" (a12) -- NCCL all-gather of x into x_full, then the local SpMV.
-    cfg = cfg_of(HEADLINE)
-    xchunk = -(-gspec.ncols // world)
-    xb = min(rank * xchunk, gspec.ncols)
-    xl = R.spmv_x(gspec, begin=xb, n=min(xchunk, gspec.ncols - xb))
-    h_xl = torch.zeros(xchunk, dtype=torch.float64).pin_memory()
-    h_xl[:xl.size] = torch.from_numpy(xl)
+    flush = torch.empty(FLUSH_BYTES, dtype=torch.uint8, device=dev)
+    chunk, rb, nloc = P.shard_rows(spec.nrows, world, rank)
+    xb, xn = P.local_x_range(spec.ncols, world, rank)
+    xc = P.x_chunk(spec.ncols, world)
+    x_full_host = R.spmv_x(spec)                      # the oracle reads global columns
+    h_xl = torch.zeros(xc, dtype=torch.float64).pin_memory()
+    h_xl[:xn] = torch.from_numpy(x_full_host[xb:xb + xn])
     d_xl = h_xl.to(dev)
+    threads = max(1, (os.cpu_count() or 1) // world)
+    drp, dcol, dval, nnz, yref, aref = gen_to_device(torch, spec, dev, row_begin=rb, nrows=nloc, with_oracle=True,
+                                                     x=x_full_host, threads=threads)
     d_y = torch.empty(nloc, dtype=torch.float64, device=dev)
-    nnz_t = torch.tensor([nnz], dtype=torch.int64, device=dev)
+    nnz_t = torch.tensor([nnz], dtype=torch.int64, device=dev if not SHARE_GPU else "cpu")
     dist.all_reduce(nnz_t)
-    B = alg_bytes(gspec.nrows, gspec.ncols, int(nnz_t.item()))
+    B = alg_bytes(spec.nrows, spec.ncols, int(nnz_t.item()))
+    B_local = nnz * 12 + (nloc + 1) * 8 + nloc * 8 + spec.ncols * 8
+    cfg = cfg_of(HEADLINE_CFG5)
+
+    def maxr(v):
+        tt = torch.tensor([v], dtype=torch.float64, device=dev if not SHARE_GPU else "cpu")
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        return float(tt.item())
 
     def timed(step, iters):
         for _ in range(args.warmup):
@@ -385,83 +515,109 @@ def run_gpu(args, rank, world, local_rank):
             ts = time_steps(torch, step, flush, P, iters)
             torch.cuda.synchronize()
         dist.barrier()
-        t = torch.tensor([sum(ts) / len(ts)], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)   # max over ranks
-        return float(t.item()), clk.summary()
+        return maxr(sum(ts) / len(ts)), clk.summary()   # max over ranks
 
-    res = {}
+    res, checks = {}, {}
     comm = None
-    y_ag = None
     if not SHARE_GPU:   # NCCL needs one GPU per rank
         comm = P.Comm()
-        d_xf = torch.empty(xchunk * world, dtype=torch.float64, device=dev)
-        res["allgather"] = timed(lambda: comm.spmv_csr_f64(gspec.nrows, gspec.ncols, d_rp, d_col, d_val, d_xl,
-                                                           d_xf, d_y, **cfg), args.steps)
-        y_ag = d_y.clone()
+        d_xf = torch.empty(xc * world, dtype=torch.float64, device=dev)
+        res["step_allgather_spmv"] = timed(lambda: comm.spmv_csr_f64(spec.nrows, spec.ncols, drp, dcol, dval, d_xl,
+                                                                     d_xf, d_y, **cfg), args.steps)
+        checks["allgather"] = parity(d_y.cpu().numpy(), yref, aref)
+        res["allgather_alone"] = timed(lambda: comm.allgather_x(d_xl, d_xf, spec.ncols), args.steps)
+        res["local_spmv_alone"] = timed(lambda: P.spmv_csr_f64(drp, dcol, dval, d_xf, d_y, ncols=spec.ncols,
+                                                               **cfg), args.steps)
     xp_err = None
     try:
-        xp = P.XPeer(gspec.ncols)
+        xp = P.XPeer(spec.ncols)
         xp.set_local_x(d_xl)
-        res["xpeer"] = timed(lambda: xp.spmv_csr_f64(gspec.nrows, d_rp, d_col, d_val, d_y, **cfg), args.steps)
-        # R16: same rows, same variant -> same bits (even nnz offsets)
-        same = bool(torch.equal(d_y, y_ag)) if y_ag is not None else None
-        # e2e through the public API: H2D of the local CSR and x slice from pinned
-        # memory, the peer-gather SpMV, D2H of y_local -- all inside the timed region
-        h_y = torch.empty(nloc, dtype=torch.float64).pin_memory()
-
-        def e2e_step():
-            a = h_rp.to(dev, non_blocking=True)
-            c = h_col.to(dev, non_blocking=True)
-            v = h_val.to(dev, non_blocking=True)
-            xl_d = h_xl.to(dev, non_blocking=True)
-            xp.set_local_x(xl_d)
-            h_y.copy_(xp.spmv_csr_f64(gspec.nrows, a, c, v, **cfg), non_blocking=True)
-        ms_e2e, _ = timed(e2e_step, max(3, args.steps // 20))
-        e2e = {"value": B / (ms_e2e / 1e3) / 1e9, "unit": UNIT, "ms_per_step": ms_e2e,
-               "h2d_bytes_per_step": (h_rp.numel() + h_col.numel() // 2 + h_val.numel() + h_xl.numel()) * 8,
-               "d2h_bytes_per_step": nloc * 8}
-    except P.NestError as e:   # reported, and the all-gather number stands in
-        xp_err, same, e2e = str(e), None, None
-    head = "xpeer" if "xpeer" in res else "allgather"
+        res["step_peer_gather"] = timed(lambda: xp.spmv_csr_f64(spec.nrows, drp, dcol, dval, d_y, **cfg),
+                                        args.steps)
+        checks["peer_gather"] = parity(d_y.cpu().numpy(), yref, aref)
+    except P.NestError as e:
+        xp, xp_err = None, str(e)
+    head = "step_allgather_spmv" if "step_allgather_spmv" in res else "step_peer_gather"
     ms, clocks = res[head]
+    worst = maxr(max(c["worst_rel_to_abs"] for c in checks.values()))
+
+    # e2e through the public API with HOST buffers: the shard and x slice cross PCIe,
+    # all-gather + local SpMV, y_local back (a12 hostio entry point)
+    e2e = None
+    if comm is not None:
+        cpu = lambda a: a.cpu().pin_memory()
+        h_rp, h_col, h_val, h_y = cpu(drp), cpu(dcol), cpu(dval), torch.empty(nloc, dtype=torch.float64).pin_memory()
+        ws = torch.empty(comm.hostio_workspace_bytes(nloc, nnz, spec.ncols), dtype=torch.uint8, device=dev)
+        del drp, dcol, dval
+        torch.cuda.empty_cache()
+        ms_e2e, _ = timed(lambda: comm.spmv_csr_f64_hostio(spec.nrows, spec.ncols, h_rp, h_col, h_val, h_xl, h_y,
+                                                            ws, **cfg), max(3, min(args.steps, 5)))
+        e2e = {"value": B / (ms_e2e / 1e3) / 1e9, "unit": UNIT, "ms_per_step": ms_e2e,
+               "h2d_bytes_per_step": (nloc + 1) * 8 + nnz * 12 + xc * 8, "d2h_bytes_per_step": nloc * 8,
+               "note": "per rank; nest_spmv_csr_f64_dist_hostio, max over ranks"}
     if rank == 0:
+        ag_bytes = (world - 1) * xc * 8
         line = {"metric": METRIC, "value": B / (ms / 1e3) / 1e9, "unit": UNIT, "n_gpus": world,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
-                "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-                "config": {"workload": f"row-partitioned CSR SpMV fp64, {spec.nrows} rows per rank "
-                                       f"(global {gspec.nrows}), nnz/row U{{{spec.nnz_min}..{spec.nnz_max}}}, "
-                                       f"banded+far; x exchange: {head}", "parallelism": f"rows/{world}",
-                           "l2": "flushed between timed steps", "variant": "blocked teams + 128-bit pair loads",
-                           **cfg},
-                "exchange": {k: {"ms_per_step": v[0], "GBs": B / (v[0] / 1e3) / 1e9} for k, v in res.items()},
-                "xpeer_error": xp_err, "xpeer_bitwise_equal_allgather": same,
-                "gpu_launches": args.steps * (3 if head == "xpeer" else 1),
-                "gpu_launches_detail": ("per step: barrier + SpMV + barrier kernels (+ l2_flush outside the events)"
-                                        if head == "xpeer" else "per step: SpMV kernel + NCCL all-gather"),
+                "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+                "config": {"workload": workload(spec, "configs[4], row-partitioned at fixed total size"),
+                           "alg_bytes": B, "parallelism": f"rows/{world}", "x_exchange": head,
+                           "l2": "flushed between timed steps", **cfg},
+                "parts_ms": {k: v[0] for k, v in res.items()},
+                "local_spmv_GBs_per_gpu": (B_local / (res["local_spmv_alone"][0] / 1e3) / 1e9
+                                           if "local_spmv_alone" in res else None),
+                "allgather_busbw_GBs": (ag_bytes / (res["allgather_alone"][0] / 1e3) / 1e9
+                                        if "allgather_alone" in res else None),
+                "parity": {"rows_checked": spec.nrows, "worst_rel_to_abs_over_ranks": worst,
+                           "ok": bool(worst <= 1e-12), "per_variant_rank0": checks},
+                "xpeer_error": xp_err,
+                "gpu_launches": args.steps * (3 if head == "step_allgather_spmv" else 5),
+                "gpu_launches_detail": ("per step: NCCL all-gather + SpMV kernel (+ 2 l2_flush kernels outside "
+                                        "the events)" if head == "step_allgather_spmv" else
+                                        "per step: barrier + SpMV + barrier (+ 2 l2_flush)"),
                 "clocks": clocks, "e2e": e2e}
-        peak, peak_src = peaks()
         per_gpu = line["value"] / world
         line["roofline"] = {"bound": "hbm", "achieved": per_gpu, "peak": peak, "unit": "GB/s",
                             "frac": per_gpu / peak, "traffic": None, "peak_source": peak_src,
-                            "kernel": f"nest_kernel_2pm<S={cfg['simdlen']},{cfg['mode']},SUM,U=1,SpmvVecBody<0,2,int,"
-                                      f"{'XPeer' if head == 'xpeer' else 'XLocal'}>>",
+                            "kernel": kernel_name(HEADLINE_CFG5),
                             "note": "per GPU: algorithmic bytes of all ranks / world / max-over-ranks step time"}
+        if not args.no_cpu_baseline:
+            line["cpu_baseline"] = cpu_sample_multi(spec)
         print(json.dumps(line), flush=True)
-    if "xpeer" in res:
+    if xp is not None:
         xp.close()
     if comm is not None:
         comm.close()
 
 
+def cpu_sample_multi(spec):
+    """N > 1: the oracle (1 thread) on a bounded sample of configs[4]: its first
+    5M rows (about 80M nonzeros), repeated for ~10 s."""
+    import oracle
+    n = 5_000_000
+    rp, col, val = R.spmv_matrix(spec, row_begin=0, nrows=n)
+    x = R.spmv_x(spec)
+    Bs = val.size * 12 + (n + 1) * 8 + n * 8 + spec.ncols * 8
+    passes, t_total = 0, 0.0
+    while t_total < 10.0:
+        t0 = time.perf_counter()
+        oracle.spmv_csr_f64(rp, col, val, x)
+        t_total += time.perf_counter() - t0
+        passes += 1
+    return {"value": Bs * passes / t_total / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"{passes} passes over rows [0, {n}) of {spec.name} ({val.size} nnz), single-threaded C",
+            "host": host_cpu()}
+
+
 # Developer check of the N > 1 code path on a one-GPU box: every rank on cuda:0,
-# gloo process group, the NCCL all-gather leg skipped (timings are meaningless).
+# gloo process group, the NCCL legs skipped (timings are meaningless).
 SHARE_GPU = os.environ.get("NEST_BENCH_SHARE_GPU") == "1"
 
 
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--steps", type=int, default=50)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -481,8 +637,10 @@ def main():
     try:
         if args.impl == "reference":
             run_reference(args, rank, world)
+        elif world == 1:
+            run_gpu_single(args, local_rank)
         else:
-            run_gpu(args, rank, world, local_rank)
+            run_gpu_multi(args, rank, world, local_rank)
     finally:
         if world > 1:
             import torch.distributed as dist

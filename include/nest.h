@@ -311,6 +311,24 @@ nest_status nest_spmv_csr_f64_dist(const nest_desc *desc, nest_comm *comm, int64
                                    const double *val, const double *x_local, double *x_full,
                                    double *y_local, void *stream);
 
+/* a12's exchange step on its own: ncclAllGather of every rank's x_local
+ * (xchunk doubles) into x_full (nranks*xchunk doubles) on `stream`. */
+nest_status nest_comm_allgather_x(nest_comm *comm, const double *x_local, double *x_full, int64_t xchunk,
+                                  void *stream);
+
+/* a12 end to end from HOST buffers (pinned for asynchronous copies): the rank's
+ * CSR shard (0-based rowptr_local, global colind), its x slice (xchunk doubles)
+ * are copied into `d_workspace` (device, >= nest_spmv_dist_hostio_workspace_bytes,
+ * 256-byte aligned), then nest_spmv_csr_f64_dist runs on the copies and y_local
+ * returns to h_y_local.  All validation before the first copy. */
+size_t nest_spmv_dist_hostio_workspace_bytes(int64_t nrows_local, int64_t nnz_local, int64_t xchunk,
+                                             int32_t nranks);
+nest_status nest_spmv_csr_f64_dist_hostio(const nest_desc *desc, nest_comm *comm, int64_t nrows_global,
+                                          int64_t ncols_global, int64_t nrows_local, int64_t nnz_local,
+                                          const int64_t *h_rowptr_local, const int32_t *h_colind,
+                                          const double *h_val, const double *h_x_local, double *h_y_local,
+                                          void *d_workspace, size_t workspace_bytes, void *stream);
+
 /* ---- NEXT-3: several parallel regions with their own simdlen in ONE kernel ----
  * PAPER.md:511-513 ("the size could differ between parallel regions") and
  * PAPER.md:686-698.  Every team runs regions[0..nregions) in order; region k

@@ -29,6 +29,8 @@ def lib():
         L = ctypes.CDLL(_LIB_PATH)
         i64, i32, vp = ctypes.c_int64, ctypes.c_int32, ctypes.c_void_p
         L.oracle_spmv_csr_f64.argtypes = [i64, vp, vp, vp, vp, ctypes.c_int, vp, vp]
+        L.oracle_spmv_csr_f64_threads.argtypes = [i64, vp, vp, vp, vp, ctypes.c_int, vp, vp, ctypes.c_int]
+        L.oracle_spmv_csr_f64_threads.restype = ctypes.c_int
         L.oracle_batched_matvec_f32.argtypes = [i64, i32, i32, vp, vp, ctypes.c_int, vp, vp]
         L.oracle_nested_stencil_f64.argtypes = [i64, i32, vp, vp, vp, ctypes.c_int, vp, vp, vp]
         L.oracle_group_map.argtypes = [i32, i32, vp]
@@ -65,6 +67,20 @@ def spmv_csr_f64(rowptr, col, val, x, op="sum"):
     if lib().oracle_spmv_csr_f64(n, _p(rowptr), _p(col), _p(val), _p(x), _op(op), _p(y), _p(a)):
         raise ValueError("oracle_spmv_csr_f64: bad arguments")
     return y, a
+
+
+def spmv_csr_f64_threads(rowptr, col, val, x, threads, op="sum"):
+    """a8 on `threads` host threads (OpenMP over rows, the same per-row loop):
+    bit-identical to spmv_csr_f64.  Returns (y, abs, threads actually used)."""
+    rowptr, col, val, x = _c(rowptr, np.int64), _c(col, np.int32), _c(val, np.float64), _c(x, np.float64)
+    n = rowptr.size - 1
+    y = np.empty(n, np.float64)
+    a = np.empty(n, np.float64)
+    used = lib().oracle_spmv_csr_f64_threads(n, _p(rowptr), _p(col), _p(val), _p(x), _op(op), _p(y), _p(a),
+                                             int(threads))
+    if used < 1:
+        raise ValueError("oracle_spmv_csr_f64_threads: bad arguments")
+    return y, a, used
 
 
 def batched_matvec_f32(A, x, batch, m=64, n=64, op="sum"):

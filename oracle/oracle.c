@@ -12,7 +12,9 @@
  * simd); the result it reaches is, up to
  * floating-point summation order, the plain sequential loop nest.  So each
  * body below is that loop nest written out in storage order, in fp64, compiled
- * with -O2 -ffp-contract=off (no FMA contraction, no -ffast-math).
+ * with -O2 -ffp-contract=off (no FMA contraction, no -ffast-math), on one
+ * thread -- except oracle_spmv_csr_f64_threads, the same per-row loop with the
+ * rows split among host threads (the all-cores CPU baseline; bit-identical).
  * The simd reduction is the north_star's addition (the paper used an atomic
  * update, and lists reductions as future work,
  * PAPER.md:868-873); its identity/combine are the textbook ones (R2).
@@ -28,6 +30,7 @@
  * unpinned".
  */
 #include <math.h>
+#include <omp.h>
 #include <stdint.h>
 #include <stddef.h>
 
@@ -52,20 +55,43 @@ uint32_t oracle_version(void) { return 1u; }
  *   y_i = (+)_{k in [rowptr_i, rowptr_{i+1})} val_k * x_{col_k}
  * in storage order.  absy_i = sum |val_k * x_{col_k}| (tolerance scale, R3).
  * rowptr is relative: rowptr[0] need not be 0 (entries index col/val). */
+static void spmv_row(int64_t i, const int64_t *rowptr, const int32_t *col, const double *val,
+                     const double *x, int op, double *y, double *absy) {
+    double s = or_identity(op), a = 0.0;
+    for (int64_t k = rowptr[i]; k < rowptr[i + 1]; ++k) {
+        double t = val[k] * x[col[k]];
+        s = or_combine(op, s, t);
+        a += fabs(t);
+    }
+    y[i] = s;
+    if (absy) absy[i] = a;
+}
+
 int oracle_spmv_csr_f64(int64_t nrows, const int64_t *rowptr, const int32_t *col,
                         const double *val, const double *x, int op, double *y, double *absy) {
     if (nrows < 0 || op < 0 || op > 2) return 1;
-    for (int64_t i = 0; i < nrows; ++i) {
-        double s = or_identity(op), a = 0.0;
-        for (int64_t k = rowptr[i]; k < rowptr[i + 1]; ++k) {
-            double t = val[k] * x[col[k]];
-            s = or_combine(op, s, t);
-            a += fabs(t);
-        }
-        y[i] = s;
-        if (absy) absy[i] = a;
-    }
+    for (int64_t i = 0; i < nrows; ++i) spmv_row(i, rowptr, col, val, x, op, y, absy);
     return 0;
+}
+
+/* The same per-row loop with the rows split among `nthreads` host threads
+ * (OpenMP, static schedule) -- the all-cores CPU baseline of BASELINE.md §4.
+ * Rows are independent and each row's sum runs in storage order on one thread,
+ * so the result is bit-identical to oracle_spmv_csr_f64 for any thread count
+ * (pinned by tests/test_oracle_spmv.py).  Returns the thread count used. */
+int oracle_spmv_csr_f64_threads(int64_t nrows, const int64_t *rowptr, const int32_t *col,
+                                const double *val, const double *x, int op, double *y, double *absy,
+                                int nthreads) {
+    if (nrows < 0 || op < 0 || op > 2 || nthreads < 1) return -1;
+    int used = 1;
+#pragma omp parallel num_threads(nthreads)
+    {
+#pragma omp single
+        used = omp_get_num_threads();
+#pragma omp for schedule(static)
+        for (int64_t i = 0; i < nrows; ++i) spmv_row(i, rowptr, col, val, x, op, y, absy);
+    }
+    return used;
 }
 
 /* a9 -- batched small dense matvec (SU3_bench stand-in):
@@ -122,7 +148,8 @@ int oracle_nested_stencil_f64(int64_t nouter, int32_t L, const double *in, const
 
 /* NEXT-2 -- laplace3d heat-diffusion step ("a simple
  * three-dimensional heat diffusion kernel called laplace3d"; the paper gives no
- * formula, R19 fixes the 7-point Jacobi step):
+ * formula; R21 fixes the 7-point Jacobi step, its summation order,
+ * alpha as an argument and the untouched boundary):
  *   for i in [1,nz-1), j in [1,ny-1), k in [1,nx-1):
  *     lap = (((((u[i-1][j][k] + u[i+1][j][k]) + u[i][j-1][k]) + u[i][j+1][k])
  *              + u[i][j][k-1]) + u[i][j][k+1]) - 6*u[i][j][k]

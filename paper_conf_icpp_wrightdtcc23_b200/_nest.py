@@ -83,6 +83,10 @@ SIGNATURES = {
     "nest_comm_init": (_st, [_vp, _i32, _i32, ctypes.POINTER(_vp)]),
     "nest_comm_destroy": (_st, [_vp]),
     "nest_spmv_csr_f64_dist": (_st, [_D, _vp, _i64, _i64, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _vp]),
+    "nest_comm_allgather_x": (_st, [_vp, _vp, _vp, _i64, _vp]),
+    "nest_spmv_dist_hostio_workspace_bytes": (_sz, [_i64, _i64, _i64, _i32]),
+    "nest_spmv_csr_f64_dist_hostio": (_st, [_D, _vp, _i64, _i64, _i64, _i64, _vp, _vp, _vp, _vp, _vp, _vp, _sz,
+                                            _vp]),
     "nest_region_program": (_st, [_D, ctypes.POINTER(nest_region), _i32, _vp]),
     "nest_xpeer_handle_bytes": (_sz, []),
     "nest_xpeer_create": (_st, [_i32, _i32, _i64, ctypes.POINTER(_vp), _vp]),

@@ -97,6 +97,45 @@ class Comm:
         return y_local
 
 
+    def allgather_x(self, x_local, x_full, ncols_global, *, stream=None):
+        """a12's exchange step alone: x_full = all ranks' x_local slices."""
+        torch = self._torch
+        xc = x_chunk(ncols_global, self.nranks)
+        check(N.nest_comm_allgather_x(self._h, _dev(x_local, torch.float64, xc, "x_local"),
+                                      _dev(x_full, torch.float64, xc * self.nranks, "x_full"), xc,
+                                      _stream(stream)), "nest_comm_allgather_x")
+        return x_full
+
+    def hostio_workspace_bytes(self, nrows_local, nnz_local, ncols_global) -> int:
+        return int(N.nest_spmv_dist_hostio_workspace_bytes(nrows_local, nnz_local,
+                                                           x_chunk(ncols_global, self.nranks), self.nranks))
+
+    def spmv_csr_f64_hostio(self, nrows_global, ncols_global, h_rowptr, h_colind, h_val, h_x_local, h_y,
+                            workspace, *, stream=None, **cfg):
+        """a12 end to end: HOST (pinned) shard and x slice in, y_local out."""
+        torch = self._torch
+        nrows_local = h_rowptr.numel() - 1
+        nnz = h_val.numel()
+        xc = x_chunk(ncols_global, self.nranks)
+        for t, dt, name, n in ((h_rowptr, torch.int64, "h_rowptr", nrows_local + 1),
+                               (h_colind, torch.int32, "h_colind", nnz), (h_val, torch.float64, "h_val", nnz),
+                               (h_x_local, torch.float64, "h_x_local", xc), (h_y, torch.float64, "h_y", nrows_local)):
+            if t.is_cuda or t.dtype != dt or not t.is_contiguous():
+                raise TypeError(f"{name} must be a contiguous host {dt} tensor")
+            if t.numel() < n:
+                raise ValueError(f"{name} has {t.numel()} elements, needs {n}")
+        d = make_desc(**cfg)
+        check(N.nest_spmv_csr_f64_dist_hostio(ctypes.byref(d), self._h, nrows_global, ncols_global, nrows_local, nnz,
+                                              ctypes.c_void_p(h_rowptr.data_ptr()),
+                                              ctypes.c_void_p(h_colind.data_ptr()),
+                                              ctypes.c_void_p(h_val.data_ptr()),
+                                              ctypes.c_void_p(h_x_local.data_ptr()),
+                                              ctypes.c_void_p(h_y.data_ptr()),
+                                              _dev(workspace, torch.uint8, None, "workspace"), workspace.numel(),
+                                              _stream(stream)), "nest_spmv_csr_f64_dist_hostio")
+        return h_y
+
+
 class XPeer:
     """NEXT-4: comm-free row-partitioned SpMV.  x stays distributed: this rank's
     slice lives in a libnest-owned buffer every peer maps (CUDA IPC), and the

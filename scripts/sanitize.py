@@ -18,8 +18,11 @@ for S in (2, 8, 32):
     for mode in ("spmd", "generic_smem", "generic_shfl"):
         for extra in ({}, {"blocked": True}, {"vec128": True}, {"sharing_bytes": 64}):
             P.spmv_csr_f64(rp, col, val, x, simdlen=S, mode=mode, **extra)
-        P.spmv_csr_f64(rp, col, val, x, simdlen=S, mode=mode, staged=True, x_halo=100, threads_per_team=256)
+        # x ring: copy warp + mbarrier segment ring, per-warp cp.async row-bound stages
         P.spmv_csr_f64(rp, col, val, x, simdlen=S, mode=mode, x_halo=100)
+        P.spmv_csr_f64(rp, col, val, x, simdlen=S, mode=mode, x_halo=300, vec128=True, threads_per_team=768,
+                       outer_unroll=2, num_teams=3)
+        P.spmv_csr_f64(rp[1:], col, val, x, simdlen=S, mode=mode, x_halo=50, threads_per_team=64)
         P.nested_stencil_f64(inp, coef, w, 4099, 8, simdlen=S, mode=mode)
         P.batched_matvec_f32(A, xb, 64, simdlen=S, mode=mode, outer_unroll=2)
         P.batched_matvec_f32(A, xb, 64, simdlen=S, mode=mode)   # lean SPMD / generic drivers (U = 1)

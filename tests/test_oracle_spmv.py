@@ -140,3 +140,23 @@ def test_row_shards_concatenate():
             assert np.array_equal(rpl + rp[b], rp[b:b + cnt + 1])
             parts.append(oracle.spmv_csr_f64(rpl, cl, vl, x)[0])
         assert np.array_equal(np.concatenate(parts), y)
+
+
+def test_threaded_oracle_is_bit_identical_to_the_sequential_one():
+    """The all-cores baseline runs the same per-row loop on
+    several threads: rows are independent, so any thread count gives the same
+    bits as the one-thread oracle (ragged rows, empty rows, every op)."""
+    import numpy as np
+    rng = np.random.default_rng(5)
+    lens = rng.integers(0, 40, 5003)
+    lens[::97] = 0
+    rp = np.concatenate([[0], np.cumsum(lens)]).astype(np.int64)
+    col = rng.integers(0, 3000, rp[-1]).astype(np.int32)
+    val = rng.standard_normal(rp[-1])
+    x = rng.standard_normal(3000)
+    for op in ("sum", "max", "min"):
+        y1, a1 = oracle.spmv_csr_f64(rp, col, val, x, op=op)
+        for t in (1, 2, 3, 8):
+            yt, at, used = oracle.spmv_csr_f64_threads(rp, col, val, x, t, op=op)
+            assert 1 <= used <= t
+            assert np.array_equal(y1.view(np.int64), yt.view(np.int64)) and np.array_equal(a1, at)
