@@ -23,10 +23,11 @@ namespace cg = cooperative_groups;
 
 // WU ("warp-uniform"): the caller guarantees that every lane of the warp
 // reaches each collective of the group together (all groups of the warp run
-// the same number of batches), so the data exchanges can use the full-warp
-// mask -- xor offsets < S never leave the group, results are identical --
-// and skip the sub-warp convergence checks.  Synchronisation keeps the group
-// mask (simdmask).
+// the same number of batches), so the data exchanges use the full-warp mask
+// -- xor offsets < S never leave the group, results are identical -- and skip
+// the sub-warp convergence checks, and synchronizeWarp(simdmask()) becomes a
+// full-warp __syncwarp(): with every lane of the warp at the same barrier it
+// orders exactly what the group barrier would (a superset of the group).
 template <int S, bool WU = false>
 struct SimdGroup {
     static_assert(S == 1 || S == 2 || S == 4 || S == 8 || S == 16 || S == 32,

@@ -67,17 +67,17 @@ struct RingPos {
 // x access policy of the ring (bodies.cuh XA): resident window or global gather.
 struct XRing {
     const double* x;
-    uint32_t ring;      // shared address of slot 0
-    int32_t base_c;     // first column of the round's resident window
-    uint32_t span;      // columns in the window
-    uint32_t base_pos;  // ring position (doubles) of base_c
-    uint32_t xw;        // ring capacity (doubles)
+    const double* ring;  // slot 0 of the shared-memory window
+    int32_t base_c;      // first column of the round's resident window
+    uint32_t span;       // columns in the window
+    uint32_t base_pos;   // ring position (doubles) of base_c
+    uint32_t xw;         // ring capacity (doubles)
     __device__ __forceinline__ double operator()(int32_t c) const {
         const uint32_t d = (uint32_t)(c - base_c);
         if (d < span) {
             uint32_t p = d + base_pos;
             p = p >= xw ? p - xw : p;
-            return lds_f64(ring + p * 8u);
+            return ring[p];
         }
         return __ldg(x + c);
     }
@@ -239,7 +239,7 @@ __global__ void __launch_bounds__(TPS == 2 ? 768 : 1024, TPS) spmv_ring_kernel(c
         }
         uint32_t ph_unused;
         Body b = body;   // the round's window; the rest are kernel parameters
-        b.x.ring = smem_u32(xring);
+        b.x.ring = xring;
         b.x.base_c = sA * kRingSeg;
         const int32_t cB = sB * kRingSeg < (int32_t)a.ncols ? sB * kRingSeg : (int32_t)a.ncols;
         b.x.span = (uint32_t)(cB > b.x.base_c ? cB - b.x.base_c : 0);

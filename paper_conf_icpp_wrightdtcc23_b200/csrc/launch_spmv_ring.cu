@@ -65,6 +65,9 @@ nest_status plan_spmv_ring(Plan* q, int64_t nrows, int64_t nnz, int32_t num_team
             int64_t ns = (budget - RingLayout::of(0, nc, kRingDepth, stage, sharing).total) / (kRingSeg * 8 + 16);
             while (ns > 0 && RingLayout::of((int32_t)ns, nc, kRingDepth, stage, sharing).total > budget) --ns;
             if (ns >= span + (pass == 0 ? want : 1)) {
+                // no more ring than the window plus its slack: the rest of the SM's
+                // unified L1/shared array stays L1 for the CSR stream and far gathers
+                if (pass == 0) ns = std::min<int64_t>(ns, span + 2 * want);
                 best_tps = tps, best_ns = (int32_t)ns;
                 best_total = RingLayout::of((int32_t)ns, nc, kRingDepth, stage, sharing).total;
             }
@@ -88,9 +91,14 @@ nest_status plan_spmv_ring(Plan* q, int64_t nrows, int64_t nnz, int32_t num_team
     if (num_teams > 0) {
         q->grid = num_teams;
     } else {
+        // one league of resident teams: best_tps per SM (the kernel's register budget
+        // is sized for exactly that many, __launch_bounds__)
         int64_t resident = 0;
         nest_status s = resident_blocks(T, best_total, &resident);
         if (s != NEST_OK) return s;
+        int64_t per_sm_1 = 0;
+        if ((s = resident_blocks(2048, 0, &per_sm_1)) != NEST_OK) return s;   // = the SM count
+        resident = std::min<int64_t>(resident, per_sm_1 * best_tps);
         q->grid = (int32_t)std::max<int64_t>(1, std::min(resident, rounds));
     }
     q->per_team = std::max<int64_t>(1, (nrows + q->grid - 1) / q->grid);

@@ -48,6 +48,17 @@ CONFIGS = {
         ("ring S2 pairs T768 gsmem", dict(simdlen=2, vec128=True, x_halo=4096, teams_per_sm=2, mode="generic_smem",
                                           threads_per_team=768)),
     ],
+    "diag": [
+        ("nest S2 pairs (r1 headline)", dict(simdlen=2, vec128=True, **base)),
+        ("ring S2 pairs T768 H1", dict(simdlen=2, vec128=True, x_halo=1, teams_per_sm=2, threads_per_team=768)),
+        ("ring S2 pairs T768 H4096", dict(simdlen=2, vec128=True, x_halo=4096, teams_per_sm=2, threads_per_team=768)),
+        ("ring S2 pairs T768 H1 kb4", dict(simdlen=2, vec128=True, x_halo=1, teams_per_sm=2, threads_per_team=768,
+                                           outer_unroll=4)),
+        ("ring S2 pairs T768 H4096 kb4", dict(simdlen=2, vec128=True, x_halo=4096, teams_per_sm=2,
+                                              threads_per_team=768, outer_unroll=4)),
+        ("ring S2 pairs T1024 H1 tps1", dict(simdlen=2, vec128=True, x_halo=1, teams_per_sm=1, threads_per_team=1024)),
+        ("nest S2 pairs T768", dict(simdlen=2, vec128=True, threads_per_team=768, blocked=True)),
+    ],
 }[a.configs]
 
 out = {}

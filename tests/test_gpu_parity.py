@@ -356,7 +356,7 @@ def banded():
 
 # (x_halo, rows per group per round, T, num_teams, teams_per_sm, 128-bit pairs)
 RING_CASES = ((700, 1, 256, 0, 0, False), (64, 2, 512, 0, 0, True), (4096, 4, 256, 0, 0, False),
-              (1, 1, 1024, 0, 2, True), (700, 2, 256, 5, 0, False), (3000, 1, 128, 1, 0, True),
+              (1, 1, 768, 0, 2, True), (700, 2, 256, 5, 0, False), (3000, 1, 128, 1, 0, True),
               (4096, 1, 1024, 0, 1, True), (700, 1, 64, 3, 0, False))
 
 
