@@ -43,7 +43,10 @@ struct Plan {
 // spare: fewer instructions and registers per row.
 inline bool spmv_index32(const Plan& p, int64_t nnz) {
     const int64_t lim = (int64_t)1 << 30;
-    return nnz < ((int64_t)1 << 31) - 8 && p.outer < lim && (int64_t)p.grid * p.chunk < lim;
+    // every cursor position: outer iterations, team chunk starts (grid * chunk), and
+    // the cyclic schedule's group ids and strides (grid * groups) -- ADVICE r1
+    return nnz < ((int64_t)1 << 31) - 8 && p.outer < lim && (int64_t)p.grid * p.chunk < lim &&
+           (int64_t)p.grid * p.groups < lim;
 }
 
 // Record a thread-local error message and return `s`.

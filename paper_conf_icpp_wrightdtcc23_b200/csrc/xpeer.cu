@@ -272,10 +272,12 @@ NEST_API nest_status nest_spmv_csr_f64_xpeer(const nest_desc* desc, nest_xpeer* 
             body.nnz = nnz;
             s = dispatch(p, body, fb, st);
         }
-        if (s != NEST_OK) return s;
     }
-    // nobody overwrites its slice while a peer may still read it
-    return nest_xpeer_barrier(xp, stream);
+    // nobody overwrites its slice while a peer may still read it.  Posted even when
+    // the launch failed (e.g. the variant's thread limit), so every rank's barrier
+    // epochs stay in step and no peer waits for an epoch this rank never posts.
+    const nest_status sb = nest_xpeer_barrier(xp, stream);
+    return s != NEST_OK ? s : sb;
 }
 
 NEST_API nest_status nest_xpeer_destroy(nest_xpeer* xp) {

@@ -224,3 +224,13 @@ def test_spmv_plan_x_ring_rejections():
     with pytest.raises(P.NestError) as e:    # the removed staged-pipeline bit is an unknown flag
         P.spmv_plan(1000, 1000, 8000, flags=1 << 2, num_teams=1)
     assert e.value.status == N.NEST_ERR_INVALID_ARG
+
+
+def test_spmv_plan_index_width_covers_the_cyclic_schedule():
+    """32-bit cursors only when grid * G (the cyclic schedule's group
+    ids and stride) also stays below 2^30 -- a caller-set league of 3M teams of
+    1024 lanes at simdlen 1 would overflow them."""
+    small = P.spmv_plan(1000, 1000, 8000, simdlen=1, threads_per_team=1024, num_teams=100)
+    assert small["index_bits"] == 32
+    big = P.spmv_plan(1000, 1000, 8000, simdlen=1, threads_per_team=1024, num_teams=3_000_000)
+    assert big["index_bits"] == 64
