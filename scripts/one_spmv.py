@@ -1,12 +1,16 @@
-"""Run one SpMV variant a few times (for ncu captures).  Usage:
-python scripts/one_spmv.py --spec CFG2 --S 8 --mode spmd --U 1 --hints 0 --iters 3"""
+"""Run one SpMV variant a few times (for ncu captures).  The matrix is generated
+in row chunks straight into device memory (bench.gen_to_device), so configs[4]
+(100M rows) fits.  Usage:
+python scripts/one_spmv.py --spec CFG2 --S 2 --T 1024 --blocked 1 --vec 1 --iters 3"""
 import argparse
 import os
 import sys
 
 import torch
 
-sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import bench  # noqa: E402
 import paper_conf_icpp_wrightdtcc23_b200 as P  # noqa: E402
 from nestgen import recipes as R  # noqa: E402
 
@@ -30,16 +34,15 @@ spec = getattr(R, a.spec)
 if a.far_den:
     import dataclasses
     spec = dataclasses.replace(spec, name=f"{spec.name}_far{a.far_den}", far_den=a.far_den)
-rp, col, val = R.spmv_matrix(spec)
-x = R.spmv_x(spec)
-t = [torch.from_numpy(v).cuda() for v in (rp, col, val, x)]
+drp, dcol, dval, nnz, _, _ = bench.gen_to_device(torch, spec, torch.device("cuda"))
+t = [drp, dcol, dval, torch.from_numpy(R.spmv_x(spec)).cuda()]
 y = torch.empty(spec.nrows, dtype=torch.float64, device="cuda")
 flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
 for _ in range(a.iters):
     torch.cuda.synchronize()
     P.l2_flush(flush)
     P.spmv_csr_f64(*t, y, simdlen=a.S, mode=a.mode, outer_unroll=a.U, stream_hints=bool(a.hints),
-                   threads_per_team=a.T, persistent=bool(a.persistent), x_halo=a.halo, teams_per_sm=a.tps, blocked=bool(a.blocked), vec128=a.vec >= 1, quad=a.vec == 2,
-                   team_chunk=a.chunk)
+                   threads_per_team=a.T, persistent=bool(a.persistent), x_halo=a.halo, teams_per_sm=a.tps,
+                   blocked=bool(a.blocked), vec128=a.vec >= 1, quad=a.vec == 2, team_chunk=a.chunk)
 torch.cuda.synchronize()
 print("done")

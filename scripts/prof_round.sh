@@ -1,13 +1,25 @@
-# Round profile: launch list of the bench command + full capture of the headline kernel
-# (only the compact exports come back: raw csv + summaries).
-mkdir -p gpurun_out/prof
-ncu --metrics gpu__time_duration.sum --clock-control none -c 3000 --csv --log-file gpurun_out/prof/launches.csv \
-    python bench.py --steps 20 --warmup 3 --no-cpu-baseline > gpurun_out/prof/bench_under_ncu.log 2>&1
-for v in "2 best" "1 s1"; do
-  set -- $v
-  ncu --set full --clock-control none --import-source on -k regex:nest_kernel -s 3 -c 1 \
-      -o /tmp/$2 -f python scripts/one_spmv.py --S $1 --mode spmd --U 1 --T 1024 --blocked 1 --vec 1 --iters 5 > gpurun_out/prof/$2.log 2>&1
-  ncu -i /tmp/$2.ncu-rep --page raw --csv > gpurun_out/prof/$2_raw.csv 2>/dev/null
-  python scripts/ncu_summary.py /tmp/$2.ncu-rep > gpurun_out/prof/$2_summary.txt 2>&1
-done
-python scripts/launch_summary.py gpurun_out/prof/launches.csv > gpurun_out/prof/launches_summary.txt 2>&1
+# Round profile (run under gpurun): the launch list of the bench command, and one
+# ncu --set full capture per (workload, configuration) the bench line reports --
+# its roofline "traffic" comes from these (scripts/traffic_json.py).  Only the
+# compact exports come back: raw csv pages + summaries.
+O=gpurun_out/prof; mkdir -p $O
+make host >/dev/null 2>&1
+ncu --metrics gpu__time_duration.sum --clock-control none -c 4000 --csv --log-file $O/launches.csv \
+    python bench.py --steps 20 --warmup 3 --no-cpu-baseline > $O/bench_under_ncu.log 2>&1
+python scripts/launch_summary.py $O/launches.csv > $O/launches_summary.txt 2>&1
+# tag spec S T blocked vec halo tps kernel-regex
+while read tag spec S T B V H TPS K; do
+  ncu --set full --clock-control none --import-source on -k regex:$K -s 2 -c 1 -o /tmp/$tag -f \
+      python scripts/one_spmv.py --spec $spec --S $S --mode spmd --U 1 --T $T --blocked $B --vec $V --halo $H \
+      --tps $TPS --iters 3 > $O/$tag.log 2>&1
+  ncu -i /tmp/$tag.ncu-rep --page raw --csv > $O/${tag}_raw.csv 2>/dev/null
+  python scripts/ncu_summary.py /tmp/$tag.ncu-rep > $O/${tag}_summary.txt 2>&1
+done <<'LIST'
+cfg2_S2bv CFG2 2 1024 1 1 0 0 nest_kernel
+cfg2_S1bv CFG2 1 1024 1 1 0 0 nest_kernel
+g100_S2bv G100 2 1024 1 1 0 0 nest_kernel
+g100_S1bv G100 1 1024 1 1 0 0 nest_kernel
+cfg5_S8bv CFG5 8 1024 1 1 0 0 nest_kernel
+cfg5_S1bv CFG5 1 1024 1 1 0 0 nest_kernel
+cfg2_ring_S2v CFG2 2 768 0 1 4096 2 spmv_ring
+LIST

@@ -25,11 +25,11 @@ ap.add_argument("--check", action="store_true")
 ap.add_argument("--configs", default="default")
 a = ap.parse_args()
 spec = getattr(R, a.spec)
-rp, col, val = R.spmv_matrix(spec)
+import bench  # noqa: E402
 x = R.spmv_x(spec)
-nnz = val.size
+drp, dcol, dval, nnz, _, _ = bench.gen_to_device(torch, spec, torch.device("cuda"))
 B = nnz * 12 + (spec.nrows + 1) * 8 + spec.nrows * 8 + spec.ncols * 8
-t = [torch.from_numpy(v).cuda() for v in (rp, col, val, x)]
+t = [drp, dcol, dval, torch.from_numpy(x).cuda()]
 flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
 
 base = dict(threads_per_team=1024, blocked=True)
@@ -48,6 +48,12 @@ CONFIGS = {
         ("ring S2 pairs T768 gsmem", dict(simdlen=2, vec128=True, x_halo=4096, teams_per_sm=2, mode="generic_smem",
                                           threads_per_team=768)),
     ],
+    "chunks": [(f"S{S} {'pairs' if v else 'scalar'} chunk {c}",
+                dict(simdlen=S, vec128=v, team_chunk=c, **base))
+               for S, v in ((8, True), (4, True), (2, True), (1, True), (8, False))
+               for c in (0, 512, 2048, 8192, 32768)],
+    "hint": [("S8 pairs", dict(simdlen=8, vec128=True, **base)), ("S2 pairs", dict(simdlen=2, vec128=True, **base)),
+             ("S4 pairs", dict(simdlen=4, vec128=True, **base)), ("S1 pairs", dict(simdlen=1, vec128=True, **base))],
     "diag": [
         ("nest S2 pairs (r1 headline)", dict(simdlen=2, vec128=True, **base)),
         ("ring S2 pairs T768 H1", dict(simdlen=2, vec128=True, x_halo=1, teams_per_sm=2, threads_per_team=768)),
