@@ -168,8 +168,13 @@ def laplace(out):
             for blocked in (False, True):
                 for T in (256, 1024):
                     for vec in (False, True):   # scalar points / aligned pairs (LaplaceVecBody)
-                        ms = timed(lambda: P.laplace3d_f64(u, o, nz, ny, nx, 0.1, simdlen=S, mode=mode,
-                                                           blocked=blocked, threads_per_team=T, vec128=vec), iters=7)
+                        try:
+                            ms = timed(lambda: P.laplace3d_f64(u, o, nz, ny, nx, 0.1, simdlen=S, mode=mode,
+                                                               blocked=blocked, threads_per_team=T, vec128=vec),
+                                       iters=7)
+                        except P.NestError as e:   # e.g. T above the variant's register limit
+                            print("skip laplace", S, mode, blocked, T, vec, str(e)[:60])
+                            continue
                         res.append(dict(S=S, mode=mode, blocked=blocked, T=T, vec=vec, ms=ms, GBs=B / ms / 1e6))
     # Fig 10 (time over No-SIMD at S = 32) on the scalar simd unit, as in the paper
     sc = [r for r in res if not r["vec"]]

@@ -23,3 +23,14 @@ cfg5_S8bv CFG5 8 1024 1 1 0 0 nest_kernel
 cfg5_S1bv CFG5 1 1024 1 1 0 0 nest_kernel
 cfg2_ring_S2v CFG2 2 768 0 1 4096 2 spmv_ring
 LIST
+# per-instruction source pages of the headline and the S = 4 / 8 cfg2 kernels (wavefront attribution)
+for v in "cfg2_S4bv 4" "cfg2_S8bv 8"; do
+  set -- $v
+  ncu --set full --clock-control none --import-source on -k regex:nest_kernel -s 2 -c 1 -o /tmp/$1 -f \
+      python scripts/one_spmv.py --spec CFG2 --S $2 --mode spmd --U 1 --T 1024 --blocked 1 --vec 1 --iters 3 > $O/$1.log 2>&1
+  ncu -i /tmp/$1.ncu-rep --page raw --csv > $O/${1}_raw.csv 2>/dev/null
+  python scripts/ncu_summary.py /tmp/$1.ncu-rep > $O/${1}_summary.txt 2>&1
+done
+for t in cfg2_S2bv cfg2_S4bv cfg2_S8bv; do
+  ncu -i /tmp/$t.ncu-rep --page source --csv --print-source sass > $O/${t}_sass.csv 2>/dev/null
+done
