@@ -111,6 +111,21 @@ def test_spmv_cfg1_all_modes(P, cfg1, S, U):
             assert np.array_equal(bits(y), bits(first)), f"mode/hints {k} differs bitwise"
 
 
+@pytest.mark.parametrize("S", SIMDLENS)
+def test_spmv_transpose_reduce_is_the_butterfly(P, cfg1, S):
+    """SPMD with U loops in flight reduces all of them at once (engine.cuh
+    transpose_reduce): the same pairs in the same order as the butterfly, so real
+    results are bit-identical to U = 1 -- for SUM, MAX and MIN."""
+    rp, col, val, x, _, _ = cfg1["real"]
+    t = [dev(rp), dev(col), dev(val), dev(x)]
+    for op in ("sum", "max", "min"):
+        y1 = host(P.spmv_csr_f64(*t, simdlen=S, reduce=op, outer_unroll=1))
+        for U in (2, 4):
+            for T, blocked in ((256, False), (1024, True), (64, False)):
+                y = host(P.spmv_csr_f64(*t, simdlen=S, reduce=op, outer_unroll=U, threads_per_team=T, blocked=blocked))
+                assert np.array_equal(bits(y), bits(y1)), (op, U, T)
+
+
 def test_spmv_unroll_and_simdlen_integer_invariance(P, cfg1):
     rp, col, val, x, yref, _ = cfg1["int"]
     t = [dev(rp), dev(col), dev(val), dev(x)]
