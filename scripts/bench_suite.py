@@ -84,10 +84,17 @@ def cfg3(out):
                     continue
                 for blocked in (False, True):
                     for vec in (False, True):   # scalar simd unit / 128-bit pairs (StencilVecBody)
-                        ms = timed_graph(lambda: P.nested_stencil_f64(*t, N, L, o, simdlen=S, mode=mode,
-                                                                      blocked=blocked, threads_per_team=256,
-                                                                      vec128=vec))
-                        res.append(dict(L=L, S=S, mode=mode, blocked=blocked, vec=vec, ms=ms, GBs=B / ms / 1e6))
+                        # SPMD at S >= 8: also 2 / 4 outer iterations per group in flight,
+                        # reduced together (transpose-reduce)
+                        for U in ((1, 2, 4) if mode == "spmd" and S >= 8 else (1,)):
+                            try:
+                                ms = timed_graph(lambda: P.nested_stencil_f64(*t, N, L, o, simdlen=S, mode=mode,
+                                                                              blocked=blocked, threads_per_team=256,
+                                                                              vec128=vec, outer_unroll=U))
+                            except P.NestError:
+                                continue
+                            res.append(dict(L=L, S=S, mode=mode, blocked=blocked, vec=vec, U=U, ms=ms,
+                                            GBs=B / ms / 1e6))
         print("cfg3 L", L, "done", flush=True)
     summary = {}
     for L in R.STENCIL_LS:
@@ -100,7 +107,7 @@ def cfg3(out):
         s1_scalar = min((r for r in rows if r["S"] == 1), key=lambda r: r["ms"])
         ratios = {}
         for S in (2, 4, 8, 16, 32):
-            sp = min((r["ms"] for r in rows if r["S"] == S and r["mode"] == "spmd"))
+            sp = min((r["ms"] for r in rows if r["S"] == S and r["mode"] == "spmd" and r["U"] == 1))
             ratios[S] = {m: min(r["ms"] for r in rows if r["S"] == S and r["mode"] == m) / sp
                          for m in ("generic_smem", "generic_shfl")}
         # honest HBM numbers: the best and the best simdlen-1 configuration again, one launch
@@ -113,7 +120,7 @@ def cfg3(out):
         for r in (best, s1):
             r["ms_flushed"] = timed(lambda: P.nested_stencil_f64(*t, N, L, o, simdlen=r["S"], mode=r["mode"],
                                                                  blocked=r["blocked"], threads_per_team=256,
-                                                                 vec128=r["vec"]), iters=20)
+                                                                 vec128=r["vec"], outer_unroll=r["U"]), iters=20)
             r["GBs_flushed"] = B / r["ms_flushed"] / 1e6
         summary[L] = dict(best=best, simdlen1=s1, speedup_vs_simdlen1=s1["ms"] / best["ms"],
                           speedup_vs_simdlen1_flushed=s1["ms_flushed"] / best["ms_flushed"],
@@ -309,15 +316,19 @@ def fig9(out):
         for S in (1, 2, 4, 8, 16, 32):
             for mode in (("spmd",) if S == 1 else MODES):
                 best = None
-                for flags in ("b", "bv", "bq"):
-                    cfg = dict(simdlen=S, mode=mode, threads_per_team=1024, blocked=True, vec128=flags != "b",
-                               quad=flags == "bq")
+                # U > 1 in SPMD: U rows per group in flight, reduced together (transpose-reduce)
+                variants = [(f, 1, 1024) for f in ("b", "bv", "bq")]
+                if mode == "spmd" and S > 1:
+                    variants += [(f, U, T) for f in ("b", "bv") for U in (2, 4) for T in (512, 1024)]
+                for flags, U, T in variants:
+                    cfg = dict(simdlen=S, mode=mode, threads_per_team=T, blocked=True, vec128=flags != "b",
+                               quad=flags == "bq", outer_unroll=U)
                     try:
                         ms = timed(lambda: P.spmv_csr_f64(*t, y, **cfg), iters=5)
                     except P.NestError:
                         continue
                     if best is None or ms < best["ms"]:
-                        best = dict(S=S, mode=mode, variant=flags, ms=ms, GBs=B / ms / 1e6)
+                        best = dict(S=S, mode=mode, variant=flags, U=U, T=T, ms=ms, GBs=B / ms / 1e6)
                 rows.append(best)
         s1 = rows[0]["ms"]
         for r in rows:
