@@ -173,6 +173,7 @@ struct SpmvBody {
     static __device__ __forceinline__ Loop loop_of(int64_t b, int64_t e) { return Loop{(I)(e - b), (I)b}; }
 
     static __device__ __forceinline__ int steps(const SpmvBody&) { return 1; }
+    static constexpr bool kOneStep = true;
     static __device__ __forceinline__ void team_begin(TeamShared&) {}
     static __device__ __forceinline__ void team_end(const SpmvBody&, TeamShared&) {}
 
@@ -255,6 +256,7 @@ struct SpmvVecBody {
     int64_t nnz;
 
     static __device__ __forceinline__ int steps(const SpmvVecBody&) { return 1; }
+    static constexpr bool kOneStep = true;
     static __device__ __forceinline__ void team_begin(TeamShared&) {}
     static __device__ __forceinline__ void team_end(const SpmvVecBody&, TeamShared&) {}
 
@@ -505,6 +507,7 @@ struct StencilBody {
     int32_t L;
 
     static __device__ __forceinline__ int steps(const StencilBody&) { return 1; }
+    static constexpr bool kOneStep = true;
     static __device__ __forceinline__ void team_begin(TeamShared& t) {
         if (threadIdx.x == 0) t.visits = 0ull;
     }

@@ -54,6 +54,9 @@ CONFIGS = {
                for c in (0, 512, 2048, 8192, 32768)],
     "hint": [("S8 pairs", dict(simdlen=8, vec128=True, **base)), ("S2 pairs", dict(simdlen=2, vec128=True, **base)),
              ("S4 pairs", dict(simdlen=4, vec128=True, **base)), ("S1 pairs", dict(simdlen=1, vec128=True, **base))],
+    "unroll": [(f"S{S} {'pairs' if v else 'scalar'} U{U} T{T}", dict(simdlen=S, vec128=v, outer_unroll=U,
+                                                                    threads_per_team=T, blocked=True))
+               for S in (2, 4, 8, 16) for v in (True, False) for U in (1, 2, 4) for T in (512, 1024)],
     "diag": [
         ("nest S2 pairs (r1 headline)", dict(simdlen=2, vec128=True, **base)),
         ("ring S2 pairs T768 H1", dict(simdlen=2, vec128=True, x_halo=1, teams_per_sm=2, threads_per_team=768)),
