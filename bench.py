@@ -217,7 +217,8 @@ def run_reference(args, rank, world):
 # ---------------------------------------------------------------- GPU arm
 # (simdlen, mode, outer_unroll, threads_per_team, x_halo, flags) -- flags: "b" blocked
 # team schedule, "v" 128-bit pair loads, "q" 128-bit quad loads, "h" streaming cache
-# hints; x_halo > 0 is the x ring (teams_per_sm chosen by the planner)
+# hints; x_halo > 0 is the x ring (teams_per_sm chosen by the planner); SPMD with
+# outer_unroll > 1 reduces its U rows together (transpose-reduce)
 CANDIDATES = [
     (1, "spmd", 1, 256, 0, ""),
     (1, "spmd", 1, 1024, 0, "bv"),
@@ -231,9 +232,10 @@ CANDIDATES = [
     (4, "spmd", 1, 1024, 0, "bq"),
     (4, "generic_smem", 1, 1024, 0, "b"),
     (8, "spmd", 1, 1024, 0, "bv"),
+    (8, "spmd", 2, 1024, 0, "bv"),
     (8, "generic_smem", 1, 1024, 0, "b"),
-    (16, "spmd", 1, 1024, 0, "b"),
-    (32, "spmd", 1, 1024, 0, "b"),
+    (16, "spmd", 2, 1024, 0, "b"),
+    (32, "spmd", 4, 1024, 0, "b"),
     (2, "spmd", 2, 768, 4096, "v"),
 ]
 
