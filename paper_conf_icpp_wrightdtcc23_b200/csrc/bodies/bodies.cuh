@@ -563,6 +563,43 @@ struct StencilVecBody : StencilBody {
         acc = Red<OP, double>::accum(acc, c.x, t0);
         return Red<OP, double>::accum(acc, c.y, t1);
     }
+    // The lane's first H pairs (t = id, id + S, ...) as one block (engine.cuh head_iters,
+    // U = 1).  Their loads are predicated on the STATIC length L/2, not on the loop's
+    // trip count, so they do not wait for w[i] (the prologue's load that decides trip
+    // = 0 for w == 0): the in / coef loads of an outer iteration issue together with
+    // its w load -- one memory latency per outer iteration instead of two.  Loads of
+    // a skipped row are issued and discarded (they are within in[0 .. N*L+2), counted
+    // in the algorithmic bytes); the folds run only for t < trip, in t order: the
+    // per-lane order of accum, so results are bit-identical.
+    // (a head of 4 pairs at S <= 4 measured slower: L = 16/32/64 flushed 3070/4038/4578
+    // vs 3686/4352/5005 GB/s with 2)
+    static constexpr int kHeadIters = 2;
+    template <int OP, int S>
+    __device__ __forceinline__ double accum_head(const Loop& Lp, int32_t id, double acc) const {
+        constexpr int H = kHeadIters;
+        const int64_t half = L >> 1;   // pairs of the row, whatever w[i] is
+        double2 a[H], b[H], c[H];
+#pragma unroll
+        for (int h = 0; h < H; ++h) {
+            const int64_t t = id + h * S;
+            const double* p = in + Lp.base + 2 * t;
+            if (t < half) {
+                a[h] = __ldg(reinterpret_cast<const double2*>(p - 1));
+                b[h] = __ldg(reinterpret_cast<const double2*>(p + 1));
+                c[h] = __ldg(reinterpret_cast<const double2*>(coef + 2 * t));
+            }
+        }
+#pragma unroll
+        for (int h = 0; h < H; ++h) {
+            if (id + h * S < Lp.trip) {
+                const double t0 = (a[h].x + 2.0 * a[h].y) + b[h].x;
+                const double t1 = (a[h].y + 2.0 * b[h].x) + b[h].y;
+                acc = Red<OP, double>::accum(acc, c[h].x, t0);
+                acc = Red<OP, double>::accum(acc, c[h].y, t1);
+            }
+        }
+        return acc;
+    }
 };
 
 // ------------------------------------------------ NEXT-2 laplace3d
