@@ -5,7 +5,7 @@
 
 N = 1: one step = one y = A x over BASELINE.json configs[1] (10M x 10M CSR,
 nnz/row U{4..12} banded+far, fp64) through the C ABI in the headline
-configuration (simdlen 2, SPMD, blocked teams, 128-bit pairs); ``value`` is its
+configuration (simdlen 2, SPMD, blocked teams, quad tuples); ``value`` is its
 algorithmic GB/s.  The same line carries the simd-folded two-level mapping
 (simdlen 1) timed the same way, a short sweep of (simdlen, mode, variant), the
 north_star's 100M-nnz gate matrix (G100) and configs[4] on one GPU (100M rows,
@@ -241,8 +241,9 @@ CANDIDATES = [
 
 # The headline: the best measured THREE-level configuration (simdlen >= 2; the
 # metric is the 3-level mapping's GB/s): simdlen 2, SPMD, blocked teams of 1024,
-# 128-bit pair loads.  The 2-level comparison point is the best simdlen-1 candidate.
-HEADLINE = (2, "spmd", 1, 1024, 0, "bv")
+# quads of nonzeros (one 128-bit colind + one 256-bit val load per lane).  The
+# 2-level comparison point is the best simdlen-1 candidate.
+HEADLINE = (2, "spmd", 1, 1024, 0, "bq")
 SIMDLEN1 = [c for c in CANDIDATES if c[0] == 1]
 # configs[4] (16 nnz/row): wider groups pay (DESIGN.md Fig 9 analogue / cfg5 table)
 HEADLINE_CFG5 = (8, "spmd", 1, 1024, 0, "bv")

@@ -111,7 +111,8 @@ enum {
      * val and 8-byte aligned colind. */
     NEST_F_VEC128 = 1u << 4,
     /* with NEST_F_VEC128: quads instead of pairs (one 128-bit colind load and
-     * two 128-bit val loads per lane iteration); needs 16-byte aligned colind. */
+     * one 256-bit val load per lane iteration); needs 16-byte aligned colind and
+     * 32-byte aligned val. */
     NEST_F_VEC_QUAD = 1u << 5
 };
 

@@ -361,11 +361,12 @@ static nest_status spmv_launch(const Plan& p, int32_t kernel, int64_t nrows, int
 static nest_status spmv_alignment(const Plan& p, int32_t kernel, const int64_t* rowptr, const int32_t* colind,
                                   const double* val, const double* x) {
     if (reinterpret_cast<uintptr_t>(rowptr) & 7) return fail(NEST_ERR_INVALID_ARG, "rowptr must be 8-byte aligned");
+    const bool quad = (p.flags & NEST_F_VEC_QUAD) != 0;
     if ((p.flags & NEST_F_VEC128) &&
-        ((reinterpret_cast<uintptr_t>(val) & 15) ||
-         (reinterpret_cast<uintptr_t>(colind) & ((p.flags & NEST_F_VEC_QUAD) ? 15 : 7))))
-        return fail(NEST_ERR_UNSUPPORTED, "NEST_F_VEC128 needs 16-byte aligned val and %d-byte aligned colind",
-                    (p.flags & NEST_F_VEC_QUAD) ? 16 : 8);
+        ((reinterpret_cast<uintptr_t>(val) & (quad ? 31 : 15)) ||
+         (reinterpret_cast<uintptr_t>(colind) & (quad ? 15 : 7))))
+        return fail(NEST_ERR_UNSUPPORTED, "NEST_F_VEC128 needs %d-byte aligned val and %d-byte aligned colind",
+                    quad ? 32 : 16, quad ? 16 : 8);
     if (kernel == NEST_KERNEL_XRING && (reinterpret_cast<uintptr_t>(x) & 15))
         return fail(NEST_ERR_UNSUPPORTED, "x_halo needs 16-byte aligned x (bulk copies of x segments)");
     return NEST_OK;

@@ -282,12 +282,13 @@ struct SpmvVecBody {
             } else {
                 const int4 cc = HINTS ? ld_na(reinterpret_cast<const int4*>(col + k0))
                                       : __ldg(reinterpret_cast<const int4*>(col + k0));
-                const double2 v0 = HINTS ? ld_na(reinterpret_cast<const double2*>(val + k0))
-                                         : __ldg(reinterpret_cast<const double2*>(val + k0));
-                const double2 v1 = HINTS ? ld_na(reinterpret_cast<const double2*>(val + k0 + 2))
-                                         : __ldg(reinterpret_cast<const double2*>(val + k0 + 2));
                 c[0] = cc.x, c[1] = cc.y, c[2] = cc.z, c[3] = cc.w;
-                v[0] = v0.x, v[1] = v0.y, v[2] = v1.x, v[3] = v1.y;
+                // the quad's four values in ONE 256-bit load (sm_100 LDG.256; k0 is a
+                // multiple of 4, so val + k0 is 32-byte aligned): one L1 tag lookup per
+                // 32 bytes of a lane instead of two 128-bit loads
+                asm("ld.global.nc.v4.f64 {%0, %1, %2, %3}, [%4];"
+                    : "=d"(v[0]), "=d"(v[1]), "=d"(v[2]), "=d"(v[3])
+                    : "l"(val + k0));
             }
         } else if constexpr (V == 2) {   // the last entry of the arrays
             c[0] = __ldg(col + k0), v[0] = __ldg(val + k0), c[1] = c[0], v[1] = 0.0;

@@ -15,8 +15,10 @@ while read tag spec S T B V H TPS K; do
   ncu -i /tmp/$tag.ncu-rep --page raw --csv > $O/${tag}_raw.csv 2>/dev/null
   python scripts/ncu_summary.py /tmp/$tag.ncu-rep > $O/${tag}_summary.txt 2>&1
 done <<'LIST'
+cfg2_S2bq CFG2 2 1024 1 2 0 0 nest_kernel
 cfg2_S2bv CFG2 2 1024 1 1 0 0 nest_kernel
 cfg2_S1bv CFG2 1 1024 1 1 0 0 nest_kernel
+g100_S2bq G100 2 1024 1 2 0 0 nest_kernel
 g100_S2bv G100 2 1024 1 1 0 0 nest_kernel
 g100_S1bv G100 1 1024 1 1 0 0 nest_kernel
 cfg5_S8bv CFG5 8 1024 1 1 0 0 nest_kernel
@@ -31,6 +33,6 @@ for v in "cfg2_S4bv 4" "cfg2_S8bv 8"; do
   ncu -i /tmp/$1.ncu-rep --page raw --csv > $O/${1}_raw.csv 2>/dev/null
   python scripts/ncu_summary.py /tmp/$1.ncu-rep > $O/${1}_summary.txt 2>&1
 done
-for t in cfg2_S2bv cfg2_S4bv cfg2_S8bv; do
+for t in cfg2_S2bq cfg2_S2bv cfg2_S4bv cfg2_S8bv; do
   ncu -i /tmp/$t.ncu-rep --page source --csv --print-source sass > $O/${t}_sass.csv 2>/dev/null
 done

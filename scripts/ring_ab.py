@@ -59,6 +59,8 @@ CONFIGS = {
                for S in (2, 4, 8, 16) for v in (True, False) for U in (1, 2, 4) for T in (512, 1024)],
     "teams": [(f"S{S} pairs teams {nt}", dict(simdlen=S, vec128=True, num_teams=nt, **base))
               for S in (8, 2) for nt in (0, 148, 444, 592)],
+    "quads": [(f"S{S} {'quads' if q else 'pairs'}", dict(simdlen=S, vec128=True, quad=q, **base))
+              for S in (1, 2, 4, 8) for q in (False, True)],
     "diag": [
         ("nest S2 pairs (r1 headline)", dict(simdlen=2, vec128=True, **base)),
         ("ring S2 pairs T768 H1", dict(simdlen=2, vec128=True, x_halo=1, teams_per_sm=2, threads_per_team=768)),

@@ -8,8 +8,10 @@ import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 TAGS = {  # capture tag -> (spec name, bench candidate tuple)
+    "cfg2_S2bq": ("cfg2", [2, "spmd", 1, 1024, 0, "bq"]),
     "cfg2_S2bv": ("cfg2", [2, "spmd", 1, 1024, 0, "bv"]),
     "cfg2_S1bv": ("cfg2", [1, "spmd", 1, 1024, 0, "bv"]),
+    "g100_S2bq": ("g100", [2, "spmd", 1, 1024, 0, "bq"]),
     "g100_S2bv": ("g100", [2, "spmd", 1, 1024, 0, "bv"]),
     "g100_S1bv": ("g100", [1, "spmd", 1, 1024, 0, "bv"]),
     "cfg5_S8bv": ("cfg5", [8, "spmd", 1, 1024, 0, "bv"]),
