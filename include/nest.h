@@ -137,8 +137,8 @@ typedef struct {
                                  * mbarriers instead of team barriers.  Columns inside the window read
                                  * the ring, others read x in global memory: results are identical for
                                  * every H (bit-identical to nest_kernel at the same S, mode and loads).
-                                 * Needs T >= 64 and 16-byte aligned x; scalar or pair loads (not
-                                 * quads); pairs need nnz, nrows < 2^31.  0 = no ring. */
+                                 * Needs T >= 64 and 16-byte aligned x; scalar, pair or quad loads
+                                 * (tuples need nnz < 2^31); nrows < 2^31.  0 = no ring. */
     int32_t team_chunk;         /* with NEST_F_BLOCKED: outer iterations per team chunk, rounded up to
                                  * a multiple of G; team b takes chunks b, b + grid, b + 2 grid, ...
                                  * (its groups cyclically inside a chunk), so all teams sweep the

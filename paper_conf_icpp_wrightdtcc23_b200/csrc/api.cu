@@ -117,8 +117,6 @@ static nest_status plan_core(const nest_desc* d, int64_t outer, int32_t K, int32
         return fail(NEST_ERR_INVALID_ARG, "NEST_F_VEC_QUAD applies to the CSR SpMV only");
     if ((d->flags & NEST_F_VEC_QUAD) && !(d->flags & NEST_F_VEC128))
         return fail(NEST_ERR_INVALID_ARG, "NEST_F_VEC_QUAD needs NEST_F_VEC128");
-    if ((d->flags & NEST_F_VEC_QUAD) && d->x_halo > 0)
-        return fail(NEST_ERR_UNSUPPORTED, "x_halo takes scalar or pair loads (not NEST_F_VEC_QUAD)");
     if (K <= 0) K = 1;
     const int32_t S = d->simdlen;
     const bool smem_mode = d->mode == NEST_MODE_GENERIC_SMEM && S > 1;

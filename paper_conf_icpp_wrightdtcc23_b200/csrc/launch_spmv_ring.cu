@@ -12,12 +12,12 @@ constexpr int32_t kSmemPerSm = 228 * 1024;
 constexpr int32_t kSmemReservedPerBlock = 1024;
 constexpr int32_t kMaxDynSmem = 227 * 1024;
 
-enum RingBody { kScalar32, kScalar64, kPair32, kNone };
+enum RingBody { kScalar32, kScalar64, kPair32, kQuad32, kNone };
 
 RingBody ring_body(const Plan& p, int64_t nrows, int64_t nnz) {
     (void)nrows;
     const bool i32 = nnz < ((int64_t)1 << 31) - 8;
-    if (p.flags & NEST_F_VEC128) return i32 ? kPair32 : kNone;
+    if (p.flags & NEST_F_VEC128) return i32 ? ((p.flags & NEST_F_VEC_QUAD) ? kQuad32 : kPair32) : kNone;
     return i32 ? kScalar32 : kScalar64;
 }
 
@@ -26,6 +26,7 @@ int32_t ring_payload(RingBody b) {
         case kScalar32: return payload_bytes<RingScalar32, 1>();
         case kScalar64: return payload_bytes<RingScalar64, 1>();
         case kPair32: return payload_bytes<RingPair32, 1>();
+        case kQuad32: return payload_bytes<RingQuad32, 1>();
         default: return 0;
     }
 }
@@ -47,8 +48,6 @@ nest_status plan_spmv_ring(Plan* q, int64_t nrows, int64_t nnz, int32_t num_team
     if (nrows >= ((int64_t)1 << 31) - 8) return fail(NEST_ERR_UNSUPPORTED, "x_halo needs nrows < 2^31");
     const RingBody body = ring_body(*q, nrows, nnz);
     if (body == kNone) return fail(NEST_ERR_UNSUPPORTED, "x_halo with NEST_F_VEC128 needs nnz, nrows < 2^31");
-    if (q->flags & NEST_F_VEC_QUAD)
-        return fail(NEST_ERR_UNSUPPORTED, "x_halo takes scalar or pair loads (not NEST_F_VEC_QUAD)");
     const int64_t G = (int64_t)nc * 32 / S;
     const int64_t KB = q->unroll;
     const int64_t R = G * KB;
@@ -117,6 +116,7 @@ nest_status launch_spmv_ring(const Plan& p, int64_t nrows, int64_t ncols, int64_
         case kScalar32: return ring_scalar32(p, a, st);
         case kScalar64: return ring_scalar64(p, a, st);
         case kPair32: return ring_pair32(p, a, st);
+        case kQuad32: return ring_quad32(p, a, st);
         default: return fail(NEST_ERR_UNSUPPORTED, "x_halo with NEST_F_VEC128 needs nnz, nrows < 2^31");
     }
 }

@@ -60,9 +60,11 @@ nest_status ring_dispatch(const Plan& p, const RingArgs& a, cudaStream_t st) {
 using RingScalar32 = SpmvBody<false, int32_t, XRing>;
 using RingScalar64 = SpmvBody<false, int64_t, XRing>;
 using RingPair32 = SpmvVecBody<false, 2, int32_t, XRing>;
+using RingQuad32 = SpmvVecBody<false, 4, int32_t, XRing>;
 
 nest_status ring_scalar32(const Plan& p, const RingArgs& a, cudaStream_t st);
 nest_status ring_scalar64(const Plan& p, const RingArgs& a, cudaStream_t st);
 nest_status ring_pair32(const Plan& p, const RingArgs& a, cudaStream_t st);
+nest_status ring_quad32(const Plan& p, const RingArgs& a, cudaStream_t st);
 
 }  // namespace nest

@@ -61,6 +61,15 @@ CONFIGS = {
               for S in (8, 2) for nt in (0, 148, 444, 592)],
     "quads": [(f"S{S} {'quads' if q else 'pairs'}", dict(simdlen=S, vec128=True, quad=q, **base))
               for S in (1, 2, 4, 8) for q in (False, True)],
+    "ringq": [("nest S2 quads", dict(simdlen=2, vec128=True, quad=True, **base)),
+              ("ring S2 quads T768 tps2", dict(simdlen=2, vec128=True, quad=True, x_halo=4096, teams_per_sm=2,
+                                               threads_per_team=768)),
+              ("ring S2 quads T1024 tps1", dict(simdlen=2, vec128=True, quad=True, x_halo=4096, teams_per_sm=1,
+                                                threads_per_team=1024)),
+              ("ring S4 quads T768 tps2", dict(simdlen=4, vec128=True, quad=True, x_halo=4096, teams_per_sm=2,
+                                               threads_per_team=768)),
+              ("ring S2 pairs T768 tps2", dict(simdlen=2, vec128=True, x_halo=4096, teams_per_sm=2,
+                                               threads_per_team=768))],
     "diag": [
         ("nest S2 pairs (r1 headline)", dict(simdlen=2, vec128=True, **base)),
         ("ring S2 pairs T768 H1", dict(simdlen=2, vec128=True, x_halo=1, teams_per_sm=2, threads_per_team=768)),

@@ -212,9 +212,6 @@ def test_spmv_plan_x_ring_rejections():
     with pytest.raises(P.NestError) as e:    # the window cannot fit shared memory
         P.spmv_plan(1000, 1000, 8000, x_halo=200_000, num_teams=1)
     assert e.value.status == N.NEST_ERR_UNSUPPORTED
-    with pytest.raises(P.NestError) as e:    # quads are not offered with the ring
-        P.spmv_plan(1000, 1000, 8000, x_halo=100, quad=True, num_teams=1)
-    assert e.value.status == N.NEST_ERR_UNSUPPORTED
     with pytest.raises(P.NestError) as e:    # teams_per_sm only with the ring
         P.spmv_plan(1000, 1000, 8000, teams_per_sm=2, num_teams=1)
     assert e.value.status == N.NEST_ERR_INVALID_ARG

@@ -369,10 +369,10 @@ def banded():
     return out
 
 
-# (x_halo, rows per group per round, T, num_teams, teams_per_sm, 128-bit pairs)
-RING_CASES = ((700, 1, 256, 0, 0, False), (64, 2, 512, 0, 0, True), (4096, 4, 256, 0, 0, False),
-              (1, 1, 768, 0, 2, True), (700, 2, 256, 5, 0, False), (3000, 1, 128, 1, 0, True),
-              (4096, 1, 1024, 0, 1, True), (700, 1, 64, 3, 0, False))
+# (x_halo, rows per group per round, T, num_teams, teams_per_sm, tuples: 0 scalar / 2 pairs / 4 quads)
+RING_CASES = ((700, 1, 256, 0, 0, 0), (64, 2, 512, 0, 0, 2), (4096, 4, 256, 0, 0, 0),
+              (1, 1, 768, 0, 2, 2), (700, 2, 256, 5, 0, 0), (3000, 1, 128, 1, 0, 2),
+              (4096, 1, 1024, 0, 1, 2), (700, 1, 64, 3, 0, 0), (900, 1, 768, 0, 2, 4), (50, 2, 256, 7, 0, 4))
 
 
 @pytest.mark.parametrize("S", SIMDLENS)
@@ -383,10 +383,10 @@ def test_spmv_ring(P, banded, S, mode):
     for values in ("int", "real"):
         rp, col, val, x, yref, aref = banded[values]
         t = [dev(rp), dev(col), dev(val), dev(x)]
-        ynest = {vec: host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, vec128=vec)) for vec in (False, True)}
+        ynest = {v: host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, vec128=v > 0, quad=v == 4)) for v in (0, 2, 4)}
         for halo, U, T, teams, tps, vec in RING_CASES:
             cfg = dict(simdlen=S, mode=mode, outer_unroll=U, threads_per_team=T, x_halo=halo, num_teams=teams,
-                       teams_per_sm=tps, vec128=vec)
+                       teams_per_sm=tps, vec128=vec > 0, quad=vec == 4)
             assert P.spmv_plan(rp.size - 1, x.size, val.size, **cfg)["kernel"] == 1
             y = host(P.spmv_csr_f64(*t, **cfg))
             if values == "int":
@@ -432,9 +432,9 @@ def test_spmv_ring_long_rows_and_odd_sizes(P):
         for S in (1, 4, 32):
             for mode in MODES:
                 for halo, T, teams in ((3, 256, 0), (1000, 128, 0), (300, 1024, 40)):
-                    for vec in (False, True):
+                    for vec in (0, 2, 4):
                         y = host(P.spmv_csr_f64(*t, simdlen=S, mode=mode, x_halo=halo, threads_per_team=T,
-                                                num_teams=teams, vec128=vec))
+                                                num_teams=teams, vec128=vec > 0, quad=vec == 4))
                         assert np.array_equal(bits(y), bits(yref)), (lens[:3], S, mode, halo, T, vec)
 
 
@@ -461,9 +461,6 @@ def test_spmv_ring_too_big_is_unsupported(P, cfg1):
     with pytest.raises(P.NestError) as e:
         P.spmv_csr_f64(dev(rp), dev(col), dev(val), dev(x), simdlen=1, threads_per_team=1024,
                        outer_unroll=4, x_halo=20000)
-    assert e.value.status == 2
-    with pytest.raises(P.NestError) as e:   # quads are not offered with the ring
-        P.spmv_csr_f64(dev(rp), dev(col), dev(val), dev(x), x_halo=100, quad=True)
     assert e.value.status == 2
     with pytest.raises(P.NestError) as e:   # the copy warp needs a consumer warp beside it
         P.spmv_csr_f64(dev(rp), dev(col), dev(val), dev(x), x_halo=100, threads_per_team=32)
