@@ -20,7 +20,8 @@ def attrib(path):
         op = s.split()[1] if s.startswith("@") else s.split()[0]
         key = None
         if op.startswith("LDG"):
-            key = "LDG.128" if ".128" in op else ("LDG.64" if ".64" in op else "LDG.32")
+            key = ("LDG.256" if ".256" in op else "LDG.128" if ".128" in op else "LDG.64" if ".64" in op
+                   else "LDG.32")
         elif op.startswith("SHFL"):
             key = "SHFL"
         elif op.startswith("STG"):
