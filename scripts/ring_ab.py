@@ -70,6 +70,9 @@ CONFIGS = {
                                                threads_per_team=768)),
               ("ring S2 pairs T768 tps2", dict(simdlen=2, vec128=True, x_halo=4096, teams_per_sm=2,
                                                threads_per_team=768))],
+    "shape": [(f"S{S} {'quads' if q else 'pairs'} T{T}", dict(simdlen=S, vec128=True, quad=q, threads_per_team=T,
+                                                                blocked=True))
+              for S in (2, 4) for q in (True, False) for T in (256, 512, 1024)],
     "diag": [
         ("nest S2 pairs (r1 headline)", dict(simdlen=2, vec128=True, **base)),
         ("ring S2 pairs T768 H1", dict(simdlen=2, vec128=True, x_halo=1, teams_per_sm=2, threads_per_team=768)),
