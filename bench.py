@@ -634,6 +634,11 @@ def main():
         import torch.distributed as dist
         backend = "gloo" if args.impl == "reference" or SHARE_GPU else "nccl"
         if backend == "nccl":
+            # NCCL's communicator lines (one per rank, for the torch group and for
+            # libnest's own communicator) go to stderr, so the rank count is visible
+            os.environ.setdefault("NCCL_DEBUG", "INFO")
+            os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+        if backend == "nccl":
             import torch
             torch.cuda.set_device(local_rank)
         dist.init_process_group(backend)
