@@ -29,11 +29,17 @@ ap.add_argument("--blocked", type=int, default=0)
 ap.add_argument("--vec", type=int, default=0)
 ap.add_argument("--chunk", type=int, default=0)
 ap.add_argument("--far_den", type=int, default=0, help="override the spec's far-column odds (1/far_den)")
+ap.add_argument("--l2fetch", type=int, default=0, help="cudaLimitMaxL2FetchGranularity in bytes (0: default)")
 a = ap.parse_args()
 spec = getattr(R, a.spec)
 if a.far_den:
     import dataclasses
     spec = dataclasses.replace(spec, name=f"{spec.name}_far{a.far_den}", far_den=a.far_den)
+if a.l2fetch:
+    torch.cuda.init()
+    from cuda.bindings import runtime as rt
+    print("set l2 fetch", rt.cudaDeviceSetLimit(rt.cudaLimit.cudaLimitMaxL2FetchGranularity, a.l2fetch),
+          rt.cudaDeviceGetLimit(rt.cudaLimit.cudaLimitMaxL2FetchGranularity))
 drp, dcol, dval, nnz, _, _ = bench.gen_to_device(torch, spec, torch.device("cuda"))
 t = [drp, dcol, dval, torch.from_numpy(R.spmv_x(spec)).cuda()]
 y = torch.empty(spec.nrows, dtype=torch.float64, device="cuda")
