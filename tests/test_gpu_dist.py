@@ -43,6 +43,21 @@ def test_dist_spmv_single_rank_nccl():
             assert np.array_equal(y.view(np.int64), y1.view(np.int64))
         with pytest.raises(P.NestError):   # wrong local row count for the rank
             comm.spmv_csr_f64(spec.nrows + 5, spec.ncols, d[0], d[1], d[2], d[3], xf)
+        # the exchange step alone, and the host-buffer entry point
+        xf2 = torch.zeros_like(xf)
+        comm.allgather_x(d[3], xf2, spec.ncols)
+        assert torch.equal(xf2[:spec.ncols], d[3])
+        pin = lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory()
+        hy = torch.empty(spec.nrows, dtype=torch.float64).pin_memory()
+        ws = torch.empty(comm.hostio_workspace_bytes(spec.nrows, val.size, spec.ncols), dtype=torch.uint8,
+                         device="cuda")
+        for cfg in (dict(simdlen=2, quad=True, blocked=True, threads_per_team=1024), dict(simdlen=8)):
+            comm.spmv_csr_f64_hostio(spec.nrows, spec.ncols, pin(rp), pin(col), pin(val), pin(x), hy, ws, **cfg)
+            torch.cuda.synchronize()
+            y1 = P.spmv_csr_f64(*d, **cfg).cpu().numpy()
+            assert np.array_equal(hy.numpy().view(np.int64), y1.view(np.int64)), cfg
+        with pytest.raises(ValueError):    # short host buffer: refused before the C call
+            comm.spmv_csr_f64_hostio(spec.nrows, spec.ncols, pin(rp), pin(col[:-1]), pin(val), pin(x), hy, ws)
         comm.close()
     finally:
         dist.destroy_process_group()

@@ -20,11 +20,14 @@ pytestmark = pytest.mark.gpu
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
-# the bench headline, 128-bit quads, the scalar body and a generic mode
-CONFIGS = (dict(simdlen=2, threads_per_team=1024, blocked=True, vec128=True),
+# the bench headline (quads), 128-bit pairs, the scalar body, a generic mode, and the
+# x ring (chunks start at odd rows: 8-byte aligned row-bound copies)
+CONFIGS = (dict(simdlen=2, threads_per_team=1024, blocked=True, quad=True),
+           dict(simdlen=2, threads_per_team=1024, blocked=True, vec128=True),
            dict(simdlen=1, threads_per_team=1024, blocked=True, quad=True),
            dict(simdlen=8),
-           dict(simdlen=4, mode="generic_smem", threads_per_team=1024, blocked=True))
+           dict(simdlen=4, mode="generic_smem", threads_per_team=1024, blocked=True),
+           dict(simdlen=2, x_halo=300, threads_per_team=256, vec128=True))
 
 
 @pytest.fixture(scope="module")
