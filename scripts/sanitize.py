@@ -24,6 +24,11 @@ for S in (2, 8, 32):
                        outer_unroll=2, num_teams=3)
         P.spmv_csr_f64(rp[1:], col, val, x, simdlen=S, mode=mode, x_halo=50, threads_per_team=64)
         P.nested_stencil_f64(inp, coef, w, 4099, 8, simdlen=S, mode=mode)
+        # pair tuples with the speculative head; U simd loops in flight (transpose-reduce in SPMD)
+        P.nested_stencil_f64(inp, coef, w, 4099, 8, simdlen=S, mode=mode, vec128=True)
+        P.nested_stencil_f64(inp, coef, w, 4099, 8, simdlen=S, mode=mode, outer_unroll=4)
+        P.spmv_csr_f64(rp, col, val, x, simdlen=S, mode=mode, outer_unroll=2, threads_per_team=512)
+        P.spmv_csr_f64(rp, col, val, x, simdlen=S, mode=mode, quad=True, blocked=True, threads_per_team=1024)
         P.batched_matvec_f32(A, xb, 64, simdlen=S, mode=mode, outer_unroll=2)
         P.batched_matvec_f32(A, xb, 64, simdlen=S, mode=mode)   # lean SPMD / generic drivers (U = 1)
         P.spmv_csr_f64(rp, col, val, x, simdlen=S, mode=mode, blocked=True, vec128=True, threads_per_team=1024,
