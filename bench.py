@@ -217,22 +217,29 @@ def run_reference(args, rank, world):
 # ---------------------------------------------------------------- GPU arm
 # (simdlen, mode, outer_unroll, threads_per_team, x_halo, flags) -- flags: "b" blocked
 # team schedule, "v" 128-bit pair loads, "q" 128-bit quad loads, "h" streaming cache
-# hints; x_halo > 0 is the x ring (teams_per_sm chosen by the planner); SPMD with
-# outer_unroll > 1 reduces its U rows together (transpose-reduce)
+# hints, "p" x under a persisting-L2 access-policy window (NEST_F_X_L2_PERSIST); x_halo
+# > 0 is the x ring (teams_per_sm chosen by the planner); SPMD with outer_unroll > 1
+# reduces its U rows together (transpose-reduce)
 CANDIDATES = [
     (1, "spmd", 1, 256, 0, ""),
     (1, "spmd", 1, 1024, 0, "bv"),
     (1, "spmd", 1, 1024, 0, "bq"),
+    (1, "spmd", 1, 1024, 0, "bvp"),
+    (1, "spmd", 1, 1024, 0, "bqp"),
     (2, "spmd", 1, 1024, 0, "b"),
     (2, "spmd", 1, 1024, 0, "bv"),
     (2, "spmd", 1, 1024, 0, "bq"),
+    (2, "spmd", 1, 1024, 0, "bvp"),
+    (2, "spmd", 1, 1024, 0, "bqp"),
     (2, "generic_smem", 1, 1024, 0, "b"),
     (2, "generic_shfl", 1, 1024, 0, "b"),
     (4, "spmd", 1, 1024, 0, "bv"),
     (4, "spmd", 1, 1024, 0, "bq"),
+    (4, "spmd", 1, 1024, 0, "bqp"),
     (4, "generic_smem", 1, 1024, 0, "b"),
     (8, "spmd", 1, 1024, 0, "bv"),
     (8, "spmd", 2, 1024, 0, "bv"),
+    (8, "spmd", 1, 1024, 0, "bvp"),
     (8, "generic_smem", 1, 1024, 0, "b"),
     (16, "spmd", 2, 1024, 0, "b"),
     (32, "spmd", 4, 1024, 0, "b"),
@@ -243,7 +250,7 @@ CANDIDATES = [
 # metric is the 3-level mapping's GB/s): simdlen 2, SPMD, blocked teams of 1024,
 # quads of nonzeros (one 128-bit colind + one 256-bit val load per lane).  The
 # 2-level comparison point is the best simdlen-1 candidate.
-HEADLINE = (2, "spmd", 1, 1024, 0, "bq")
+HEADLINE = (2, "spmd", 1, 1024, 0, "bqp")
 SIMDLEN1 = [c for c in CANDIDATES if c[0] == 1]
 # configs[4] (16 nnz/row): wider groups pay (DESIGN.md Fig 9 analogue / cfg5 table)
 HEADLINE_CFG5 = (8, "spmd", 1, 1024, 0, "bv")
@@ -252,7 +259,8 @@ HEADLINE_CFG5 = (8, "spmd", 1, 1024, 0, "bv")
 def cfg_of(c):
     S, mode, U, T, halo, fl = c
     return dict(simdlen=S, mode=mode, outer_unroll=U, threads_per_team=T, x_halo=halo,
-                stream_hints="h" in fl, blocked="b" in fl, vec128="v" in fl or "q" in fl, quad="q" in fl)
+                stream_hints="h" in fl, blocked="b" in fl, vec128="v" in fl or "q" in fl, quad="q" in fl,
+                x_l2_persist="p" in fl)
 
 
 def cfg_key(spec, c) -> str:
@@ -267,7 +275,8 @@ def kernel_name(c) -> str:
     body = ("SpmvVecBody<0,4,int>" if "q" in fl else "SpmvVecBody<0,2,int>" if "v" in fl
             else f"SpmvBody<{int('h' in fl)},int>")
     two_pm = ("v" in fl or "q" in fl) and U == 1 and not ("q" in fl and S == 1)
-    return f"{'nest_kernel_2pm' if two_pm else 'nest_kernel'}<S={S},{mode},SUM,U={U},{body}>"
+    name = f"{'nest_kernel_2pm' if two_pm else 'nest_kernel'}<S={S},{mode},SUM,U={U},{body}>"
+    return name + (" + x persisting-L2 window" if "p" in fl else "")
 
 
 def time_steps(torch, fn, flush, P, iters):
@@ -293,6 +302,9 @@ def roofline(B, ms, peak, peak_src, c, spec):
             "traffic_source": "profiles/traffic.json: ncu --set full dram__bytes_read.sum + dram__bytes_write.sum "
                               "per launch (cold L2)",
             "traffic_over_alg_bytes": (traffic / B) if traffic else None,
+            **({"traffic_note": "ncu neutralises the persisting-L2 window (profiles/r02s3_x_l2_persist.md): this is "
+                                "the kernel's DRAM traffic WITHOUT x persisting; with it the kernel runs 5-7% faster"}
+               if "p" in c[5] else {}),
             "alg_bytes_per_launch": B,
             "alg_bytes_rule": "12 B per nonzero + 16 B per row (rowptr, y) + 8 B per column (x once)",
             "kernel": kernel_name(c), "frac_of_8TBs_spec": achieved / 8000.0}
@@ -449,7 +461,8 @@ def run_gpu_single(args, local_rank):
         "config": {"workload": workload(spec), "nnz": nnz, "alg_bytes": B, "simdlen": best[0], "mode": best[1],
                    "outer_unroll": best[2], "threads_per_team": best[3], "x_halo": best[4],
                    "variant": " + ".join({"b": "blocked teams", "h": "stream hints", "v": "128-bit pair loads",
-                                          "q": "128-bit quad loads"}[f] for f in best[5]) or "cyclic teams",
+                                          "q": "128-bit quad loads", "p": "x persisting in L2 (access-policy window)"}[f]
+                                         for f in best[5]) or "cyclic teams",
                    "l2": "flushed between timed steps (512 MiB write, then a 256 MiB read so L2 holds only clean "
                          "lines)",
                    "parallelism": "1 GPU"},

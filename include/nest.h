@@ -1,6 +1,6 @@
 /*
  * nest.h -- C ABI of the B200 three-level (teams -> parallel -> simd) loop-nest
- * library.  ABI v1.
+ * library.  ABI v2 (v2: NEST_F_X_L2_PERSIST and the nest_plan_info l2_* fields).
  *
  * What it executes (PAPER.md = /root/reference/PAPER.md, Wright et al.,
  * "Implementing OpenMP's SIMD Directive in LLVM's GPU Runtime", ICPP'23):
@@ -57,7 +57,7 @@
 extern "C" {
 #endif
 
-#define NEST_ABI_VERSION 1u
+#define NEST_ABI_VERSION 2u
 
 typedef enum {
     NEST_OK = 0,
@@ -113,7 +113,24 @@ enum {
     /* with NEST_F_VEC128: quads instead of pairs (one 128-bit colind load and
      * one 256-bit val load per lane iteration); needs 16-byte aligned colind and
      * 32-byte aligned val. */
-    NEST_F_VEC_QUAD = 1u << 5
+    NEST_F_VEC_QUAD = 1u << 5,
+    /* SpMV (nest_kernel variants: cyclic / blocked, scalar / pair / quad loads;
+     * also the dist and hostio entry points): x is marked L2-persisting for
+     * this launch.  Why: the far columns of a short-row matrix gather x at
+     * random, and with x (80-100 MB) competing against the streamed CSR arrays
+     * for the 126 MB L2 most of those gathers miss and cost a DRAM access each
+     * (DESIGN.md §6).  How: the library makes sure the device's persisting-L2
+     * set-aside (cudaLimitPersistingL2CacheSize, a DEVICE-WIDE limit; normal
+     * accesses still use it while no persisting line occupies it) is at least
+     * min(cudaDevAttrMaxPersistingL2CacheSize, 1/2 of L2), and launches the
+     * kernel with a per-launch access-policy window over x (cudaLaunchKernelEx:
+     * hitRatio = set-aside / window bytes, hits persisting, misses normal), so
+     * the caller's stream attributes are untouched.  Results are identical (a
+     * cache policy only).  The persisting lines outlive the call (a following
+     * SpMV on the same x finds them); nest_util_l2_flush returns them to
+     * normal.  With x_halo or NEST_MODE_TEAMS_GENERIC: NEST_ERR_UNSUPPORTED;
+     * other entry points: NEST_ERR_INVALID_ARG. */
+    NEST_F_X_L2_PERSIST = 1u << 6
 };
 
 /* The nest descriptor: team, thread and simd extents, mode and reduction.
@@ -173,6 +190,9 @@ typedef struct {
     int32_t ring_segments;        /* x ring: segment slots of 256 doubles (else 0) */
     int32_t ring_row_slots;       /* x ring: row-bound slots (else 0) */
     int64_t chunk;                /* blocked schedule / x ring: outer iterations per team chunk (else 0) */
+    int64_t l2_window_bytes;      /* NEST_F_X_L2_PERSIST: bytes of x under the access-policy window (else 0) */
+    int64_t l2_setaside_bytes;    /* NEST_F_X_L2_PERSIST: the persisting-L2 set-aside the launch uses (hit
+                                   * ratio = min(1, setaside / window)); else 0 */
 } nest_plan_info;
 
 uint32_t nest_abi_version(void);
@@ -283,10 +303,13 @@ nest_status nest_probe_mapping(const nest_desc *desc, int32_t *out_map, int64_t 
 nest_status nest_csr_validate(int64_t nrows, int64_t ncols, int64_t nnz, const int64_t *rowptr,
                               const int32_t *colind, int32_t *d_bad, void *stream);
 
-/* Bench utility: flush L2.  Overwrites `bytes` of device memory at `buf`, then
- * reads back its first half, so that L2 ends up holding only clean lines
- * unrelated to any later kernel (no dirty write-backs inside the next, timed,
- * kernel).  `bytes` should exceed twice the L2 size (bench: 512 MiB). */
+/* Bench utility: flush L2.  Synchronises `stream`, returns every persisting L2
+ * line of the context to normal (cudaCtxResetPersistingL2Cache: nothing a
+ * NEST_F_X_L2_PERSIST launch left behind survives), then overwrites `bytes` of
+ * device memory at `buf` and reads back its first half, so that L2 ends up
+ * holding only clean lines unrelated to any later kernel (no dirty write-backs
+ * inside the next, timed, kernel).  `bytes` should exceed twice the L2 size
+ * (bench: 512 MiB). */
 nest_status nest_util_l2_flush(void *buf, size_t bytes, void *stream);
 
 /* ---- a12: row-partitioned multi-GPU SpMV (north_star; the paper is single-GPU) ----

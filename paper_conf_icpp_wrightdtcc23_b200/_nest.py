@@ -18,7 +18,7 @@ if not os.path.exists(LIB_PATH):
                       "(there is no CPU fallback)")
 lib = ctypes.CDLL(LIB_PATH)
 
-NEST_ABI_VERSION = 1
+NEST_ABI_VERSION = 2
 NEST_OK, NEST_ERR_INVALID_ARG, NEST_ERR_UNSUPPORTED, NEST_ERR_CUDA, NEST_ERR_NCCL, NEST_ERR_NO_MEMORY = range(6)
 NEST_MODE_SPMD, NEST_MODE_GENERIC_SMEM, NEST_MODE_GENERIC_SHFL, NEST_MODE_TEAMS_GENERIC = 0, 1, 2, 3
 NEST_REDUCE_SUM, NEST_REDUCE_MAX, NEST_REDUCE_MIN = 0, 1, 2
@@ -27,6 +27,7 @@ NEST_F_STREAM_HINTS = 1 << 1
 NEST_F_BLOCKED = 1 << 3
 NEST_F_VEC128 = 1 << 4
 NEST_F_VEC_QUAD = 1 << 5
+NEST_F_X_L2_PERSIST = 1 << 6
 NEST_KERNEL_NEST, NEST_KERNEL_XRING, NEST_KERNEL_TEAMS_GENERIC = 0, 1, 2
 
 
@@ -56,7 +57,8 @@ class nest_plan_info(ctypes.Structure):
                 ("outer_unroll", ctypes.c_int32), ("smem_bytes", ctypes.c_int32),
                 ("kernel", ctypes.c_int32), ("index_bits", ctypes.c_int32),
                 ("ring_segments", ctypes.c_int32), ("ring_row_slots", ctypes.c_int32),
-                ("chunk", ctypes.c_int64)]
+                ("chunk", ctypes.c_int64), ("l2_window_bytes", ctypes.c_int64),
+                ("l2_setaside_bytes", ctypes.c_int64)]
 
 
 _i32, _i64, _u32, _vp, _sz = ctypes.c_int32, ctypes.c_int64, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_size_t

@@ -34,7 +34,7 @@ def make_desc(simdlen: int = 8, mode: str | int = "spmd", reduce: str | int = "s
               outer_unroll: int = 1, persistent: bool = False, stream_hints: bool = False,
               x_halo: int = 0, blocked: bool = False,
               vec128: bool = False, quad: bool = False, team_chunk: int = 0, teams_per_sm: int = 0,
-              flags: int = 0) -> N.nest_desc:
+              x_l2_persist: bool = False, flags: int = 0) -> N.nest_desc:
     d = N.nest_desc()
     d.abi_version = N.NEST_ABI_VERSION
     d.num_teams = num_teams
@@ -50,7 +50,7 @@ def make_desc(simdlen: int = 8, mode: str | int = "spmd", reduce: str | int = "s
     d.flags = flags | (N.NEST_F_PERSISTENT_GRID if persistent else 0) | (
         N.NEST_F_STREAM_HINTS if stream_hints else 0) | (
         N.NEST_F_BLOCKED if blocked else 0) | (N.NEST_F_VEC128 if vec128 or quad else 0) | (
-        N.NEST_F_VEC_QUAD if quad else 0)
+        N.NEST_F_VEC_QUAD if quad else 0) | (N.NEST_F_X_L2_PERSIST if x_l2_persist else 0)
     return d
 
 

@@ -4,6 +4,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <atomic>
 #include <climits>
 #include <cstdint>
 #include <cstdarg>
@@ -79,7 +80,7 @@ static nest_status validate_desc(const nest_desc* d, int32_t* T, int32_t* sharin
     if (*U != 1 && *U != 2 && *U != 4)
         return fail(NEST_ERR_INVALID_ARG, "outer_unroll %d: need 1, 2 or 4", d->outer_unroll);
     if (d->flags & ~(uint32_t)(NEST_F_PERSISTENT_GRID | NEST_F_STREAM_HINTS | NEST_F_BLOCKED |
-                               NEST_F_VEC128 | NEST_F_VEC_QUAD))
+                               NEST_F_VEC128 | NEST_F_VEC_QUAD | NEST_F_X_L2_PERSIST))
         return fail(NEST_ERR_INVALID_ARG, "unknown flags 0x%x", d->flags);
     if (d->teams_per_sm < 0 || d->teams_per_sm > 2)
         return fail(NEST_ERR_INVALID_ARG, "teams_per_sm %d: need 0, 1 or 2", d->teams_per_sm);
@@ -115,6 +116,8 @@ static nest_status plan_core(const nest_desc* d, int64_t outer, int32_t K, int32
         return fail(NEST_ERR_INVALID_ARG, "NEST_MODE_TEAMS_GENERIC applies to the CSR SpMV only");
     if ((d->flags & NEST_F_VEC_QUAD) && !spmv_window)
         return fail(NEST_ERR_INVALID_ARG, "NEST_F_VEC_QUAD applies to the CSR SpMV only");
+    if ((d->flags & NEST_F_X_L2_PERSIST) && !spmv_window)
+        return fail(NEST_ERR_INVALID_ARG, "NEST_F_X_L2_PERSIST applies to the CSR SpMV only");
     if ((d->flags & NEST_F_VEC_QUAD) && !(d->flags & NEST_F_VEC128))
         return fail(NEST_ERR_INVALID_ARG, "NEST_F_VEC_QUAD needs NEST_F_VEC128");
     if (K <= 0) K = 1;
@@ -220,6 +223,46 @@ nest_status prepare_fallback(const Plan& p, unsigned char** fb, void* stream) {
     return fallback_scratch(bytes, fb, stream);
 }
 
+// ------------------------------------------- NEST_F_X_L2_PERSIST (x in L2)
+// Set-aside the library asks for: half of L2 (63 MB on B200), capped by the
+// device's maximum persisting size (79 MB).  Measured on cfg2 / G100 (x = 80 /
+// 100 MB, profiles/r02s3_x_l2_persist.md): 63-71 MB beat 47 MB and the 79 MB
+// maximum (which leaves too little L2 for the streamed CSR lines).
+static std::mutex g_persist_mu;
+static std::map<int, int64_t> g_persist_set;   // device -> set-aside this library established
+static std::atomic<bool> g_persist_used{false};            // a persisting launch happened (nest_util_l2_flush resets)
+
+nest_status x_persist_window(Plan* p, const double* x, int64_t ncols, bool apply) {
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaGetDevice");
+    int max_persist = 0, l2 = 0, max_win = 0;
+    if ((e = cudaDeviceGetAttribute(&max_persist, cudaDevAttrMaxPersistingL2CacheSize, dev)) != cudaSuccess ||
+        (e = cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, dev)) != cudaSuccess ||
+        (e = cudaDeviceGetAttribute(&max_win, cudaDevAttrMaxAccessPolicyWindowSize, dev)) != cudaSuccess)
+        return cuda_fail(e, "cudaDeviceGetAttribute(L2 persistence)");
+    if (max_persist <= 0 || max_win <= 0)
+        return fail(NEST_ERR_UNSUPPORTED, "NEST_F_X_L2_PERSIST: the device has no persisting L2");
+    size_t cur = 0;
+    if ((e = cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize)) != cudaSuccess)
+        return cuda_fail(e, "cudaDeviceGetLimit(persisting L2)");
+    const int64_t want = std::min<int64_t>(max_persist, (int64_t)l2 / 2);
+    p->l2_win_bytes = std::min<int64_t>(ncols * 8, max_win);
+    p->l2_setaside = std::max<int64_t>((int64_t)cur, want);
+    if (!apply) return NEST_OK;
+    if ((int64_t)cur < want) {
+        std::lock_guard<std::mutex> lk(g_persist_mu);
+        if ((e = cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)want)) != cudaSuccess ||
+            (e = cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize)) != cudaSuccess)   // granularity
+            return cuda_fail(e, "cudaDeviceSetLimit(persisting L2)");
+        g_persist_set[dev] = (int64_t)cur;
+        p->l2_setaside = (int64_t)cur;
+    }
+    g_persist_used = true;
+    p->l2_win = x;
+    return NEST_OK;
+}
+
 // --------------------------------------------------------- device utilities
 __global__ void csr_validate_kernel(int64_t nrows, int64_t ncols, int64_t nnz,
                                     const int64_t* __restrict__ rowptr,
@@ -286,6 +329,8 @@ static void fill_plan_info(const Plan& p, int32_t kernel, int32_t index_bits, ne
     out->ring_segments = p.ring_nseg;
     out->ring_row_slots = p.ring_nrp;
     out->chunk = (p.flags & NEST_F_BLOCKED) || p.x_halo > 0 ? p.chunk : 0;
+    out->l2_window_bytes = p.l2_win_bytes;
+    out->l2_setaside_bytes = p.l2_setaside;
 }
 
 NEST_API nest_status nest_plan(const nest_desc* desc, int64_t outer_iters, int32_t payload_bytes,
@@ -311,7 +356,7 @@ static nest_status spmv_plan(const nest_desc* desc, int64_t nrows, int64_t ncols
     nest_status s = make_plan(desc, nrows, 1, spmv_payload, p, true);
     if (s != NEST_OK) return s;
     if (desc->mode == NEST_MODE_TEAMS_GENERIC) {
-        if ((p->flags & (NEST_F_VEC128 | NEST_F_BLOCKED)) || p->x_halo > 0)
+        if ((p->flags & (NEST_F_VEC128 | NEST_F_BLOCKED | NEST_F_X_L2_PERSIST)) || p->x_halo > 0)
             return fail(NEST_ERR_UNSUPPORTED, "NEST_MODE_TEAMS_GENERIC takes no SpMV variant flags");
         if (desc->num_teams <= 0) {
             int64_t resident = 0;
@@ -323,6 +368,8 @@ static nest_status spmv_plan(const nest_desc* desc, int64_t nrows, int64_t ncols
         return NEST_OK;
     }
     if (p->x_halo > 0) {
+        if (p->flags & NEST_F_X_L2_PERSIST)
+            return fail(NEST_ERR_UNSUPPORTED, "NEST_F_X_L2_PERSIST: not with the x ring (x_halo > 0)");
         *kernel = NEST_KERNEL_XRING;
         *index_bits = nnz < ((int64_t)1 << 31) - 8 && nrows < ((int64_t)1 << 31) - 8 ? 32 : 64;
         return plan_spmv_ring(p, nrows, nnz, desc->num_teams, desc->teams_per_sm);
@@ -331,6 +378,7 @@ static nest_status spmv_plan(const nest_desc* desc, int64_t nrows, int64_t ncols
     const int32_t payload = spmv_body_payload(*p, nnz);
     if (payload != p->payload_bytes && (s = make_plan_fixed(desc, nrows, 1, payload, p, true)) != NEST_OK) return s;
     *index_bits = spmv_index32(*p, nnz) ? 32 : 64;
+    if ((p->flags & NEST_F_X_L2_PERSIST) && (s = x_persist_window(p, nullptr, ncols, false)) != NEST_OK) return s;
     return NEST_OK;
 }
 
@@ -352,6 +400,12 @@ static nest_status spmv_launch(const Plan& p, int32_t kernel, int64_t nrows, int
                                double* y, unsigned char* fb, cudaStream_t st) {
     if (kernel == NEST_KERNEL_TEAMS_GENERIC) return launch_spmv_teams_generic(p, nrows, rowptr, colind, val, x, y, st);
     if (kernel == NEST_KERNEL_XRING) return launch_spmv_ring(p, nrows, ncols, nnz, rowptr, colind, val, x, y, fb, st);
+    if ((p.flags & NEST_F_X_L2_PERSIST) && ncols > 0) {
+        Plan q = p;
+        nest_status s = x_persist_window(&q, x, ncols, true);
+        if (s != NEST_OK) return s;
+        return launch_spmv(q, (q.flags & NEST_F_STREAM_HINTS) != 0, nrows, rowptr, colind, val, x, y, fb, st, nnz);
+    }
     return launch_spmv(p, (p.flags & NEST_F_STREAM_HINTS) != 0, nrows, rowptr, colind, val, x, y, fb, st, nnz);
 }
 
@@ -666,6 +720,13 @@ NEST_API nest_status nest_util_l2_flush(void* buf, size_t bytes, void* stream) {
     static uint32_t salt = 1;
     const size_t n16 = bytes / 16;
     if (n16 == 0) return NEST_OK;
+    if (g_persist_used) {
+        // persisting lines survive a plain flush: return them to normal first,
+        // after the work queued on `stream` (a persisting launch) has finished
+        cudaError_t e = cudaStreamSynchronize(as_stream(stream));
+        if (e == cudaSuccess) e = cudaCtxResetPersistingL2Cache();
+        if (e != cudaSuccess) return cuda_fail(e, "reset persisting L2 lines");
+    }
     l2_flush_kernel<<<1184, 512, 0, as_stream(stream)>>>(static_cast<uint4*>(buf), n16, salt++);
     l2_clean_kernel<<<1184, 512, 0, as_stream(stream)>>>(static_cast<const uint4*>(buf), n16 / 2, nullptr);
     const cudaError_t e = cudaGetLastError();

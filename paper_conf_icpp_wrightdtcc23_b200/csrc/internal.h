@@ -36,6 +36,10 @@ struct Plan {
     int32_t ring_kb = 1;         // rows per group per round (= outer_unroll)
     int32_t ring_tps = 0;        // teams per SM the ring is sized for
     int64_t per_team = 0;        // rows per team
+    // NEST_F_X_L2_PERSIST: per-launch access-policy window over x (launch_one)
+    const void* l2_win = nullptr;    // base (x); nullptr = plain launch
+    int64_t l2_win_bytes = 0;        // bytes under the window
+    int64_t l2_setaside = 0;         // persisting-L2 set-aside the hit ratio is computed from
 };
 
 // 32-bit row / nonzero indices (and 32-bit outer-loop cursors, engine.cuh
@@ -48,6 +52,12 @@ inline bool spmv_index32(const Plan& p, int64_t nnz) {
     return nnz < ((int64_t)1 << 31) - 8 && p.outer < lim && (int64_t)p.grid * p.chunk < lim &&
            (int64_t)p.grid * p.groups < lim;
 }
+
+// NEST_F_X_L2_PERSIST sizing for an x of ncols doubles on the current device:
+// window = min(x bytes, max window), set-aside = max(current limit, min(max
+// persisting, 3/8 of L2)).  apply: also raise the device's persisting-L2 limit
+// to the set-aside (once per device) and point the window at x.
+nest_status x_persist_window(Plan* p, const double* x, int64_t ncols, bool apply);
 
 // Record a thread-local error message and return `s`.
 nest_status fail(nest_status s, const char* fmt, ...) __attribute__((format(printf, 2, 3)));

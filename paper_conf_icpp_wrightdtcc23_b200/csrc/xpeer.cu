@@ -242,7 +242,7 @@ NEST_API nest_status nest_spmv_csr_f64_xpeer(const nest_desc* desc, nest_xpeer* 
     Plan p;
     nest_status s = make_plan(desc, nrows_local, 1, spmv_payload, &p, true);
     if (s != NEST_OK) return s;
-    if (desc->mode == NEST_MODE_TEAMS_GENERIC || (p.flags & NEST_F_VEC_QUAD) || p.x_halo > 0)
+    if (desc->mode == NEST_MODE_TEAMS_GENERIC || (p.flags & (NEST_F_VEC_QUAD | NEST_F_X_L2_PERSIST)) || p.x_halo > 0)
         return fail(NEST_ERR_UNSUPPORTED,
                     "nest_spmv_csr_f64_xpeer: cyclic/blocked schedules with scalar or pair loads only");
     if (nrows_local > 0 && (!rowptr || !y)) return fail(NEST_ERR_INVALID_ARG, "rowptr/y is NULL");

@@ -28,6 +28,7 @@ ap.add_argument("--tps", type=int, default=0)
 ap.add_argument("--blocked", type=int, default=0)
 ap.add_argument("--vec", type=int, default=0)
 ap.add_argument("--chunk", type=int, default=0)
+ap.add_argument("--persist", type=int, default=0, help="NEST_F_X_L2_PERSIST (x under a persisting-L2 window)")
 ap.add_argument("--far_den", type=int, default=0, help="override the spec's far-column odds (1/far_den)")
 ap.add_argument("--l2fetch", type=int, default=0, help="cudaLimitMaxL2FetchGranularity in bytes (0: default)")
 a = ap.parse_args()
@@ -49,6 +50,7 @@ for _ in range(a.iters):
     P.l2_flush(flush)
     P.spmv_csr_f64(*t, y, simdlen=a.S, mode=a.mode, outer_unroll=a.U, stream_hints=bool(a.hints),
                    threads_per_team=a.T, persistent=bool(a.persistent), x_halo=a.halo, teams_per_sm=a.tps,
-                   blocked=bool(a.blocked), vec128=a.vec >= 1, quad=a.vec == 2, team_chunk=a.chunk)
+                   blocked=bool(a.blocked), vec128=a.vec >= 1, quad=a.vec == 2, team_chunk=a.chunk,
+                   x_l2_persist=bool(a.persist))
 torch.cuda.synchronize()
 print("done")

@@ -16,6 +16,10 @@ TAGS = {  # capture tag -> (spec name, bench candidate tuple)
     "g100_S1bv": ("g100", [1, "spmd", 1, 1024, 0, "bv"]),
     "cfg5_S8bv": ("cfg5", [8, "spmd", 1, 1024, 0, "bv"]),
     "cfg5_S1bv": ("cfg5", [1, "spmd", 1, 1024, 0, "bv"]),
+    "cfg2_S2bqp": ("cfg2", [2, "spmd", 1, 1024, 0, "bqp"]),
+    "cfg2_S1bqp": ("cfg2", [1, "spmd", 1, 1024, 0, "bqp"]),
+    "g100_S2bqp": ("g100", [2, "spmd", 1, 1024, 0, "bqp"]),
+    "g100_S1bqp": ("g100", [1, "spmd", 1, 1024, 0, "bqp"]),
 }
 
 
@@ -31,14 +35,16 @@ def dram_bytes(path):
 
 
 def main(src):
-    out = {"_note": "dram__bytes_read.sum + dram__bytes_write.sum per launch, one ncu --set full capture "
+    path = os.path.join(ROOT, "profiles", "traffic.json")
+    out = json.load(open(path)) if os.path.exists(path) else {}   # keys not re-captured are kept
+    out["_note"] = ("dram__bytes_read.sum + dram__bytes_write.sum per launch, one ncu --set full capture "
                     "(--clock-control none, cold L2) per key; key = '<spec>:<bench candidate tuple>'; "
-                    f"source {src}"}
+                    f"latest source {src}")
     for tag, (spec, c) in TAGS.items():
         p = os.path.join(src, f"{tag}_raw.csv")
         if os.path.exists(p):
             out[f"{spec}:{json.dumps(c)}"] = dram_bytes(p)
-    with open(os.path.join(ROOT, "profiles", "traffic.json"), "w") as f:
+    with open(path, "w") as f:
         json.dump(out, f, indent=1)
     print(json.dumps(out, indent=1))
 

@@ -1,0 +1,513 @@
+// xgather_probe.cu -- developer micro-benchmark (not part of the library):
+// which path should the headline SpMV's x gathers take on B200?  The headline
+// (blocked teams of 1024, simdlen 2, quad tuples) sits at the L1TEX data-pipe
+// wall of its x gathers (~1 LSU wavefront per 8-byte gather).
+// Variants of the gather, everything else identical:
+//   ldg      __ldg (LDG.E.CONSTANT) -- the library's path
+//   tex      tex1Dfetch<int2> on a linear texture object (TEX pipe of L1TEX)
+//   mix      the tuple's entries 0,2 via LDG and 1,3 via TEX
+//   noX      diagnostic: no gather (col as the value) -- the floor
+// Matrix: cfg2/G100-shaped (U{4..12} nnz/row, band +-4096, 1/16 far), same
+// generator as l2x_probe.cu.  Median of 10 launches, L2 flushed before each.
+// nvcc -O3 -std=c++17 -gencode arch=compute_100a,code=sm_100a -lineinfo -o scripts/xgather_probe scripts/xgather_probe.cu
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdint>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <vector>
+
+#define CK(x)                                                                                  \
+    do {                                                                                       \
+        cudaError_t e_ = (x);                                                                  \
+        if (e_ != cudaSuccess) {                                                               \
+            fprintf(stderr, "%s:%d %s: %s\n", __FILE__, __LINE__, #x, cudaGetErrorString(e_)); \
+            exit(1);                                                                           \
+        }                                                                                      \
+    } while (0)
+
+__host__ __device__ inline uint64_t mix(uint64_t z) {
+    z += 0x9E3779B97F4A7C15ull;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+
+__global__ void gen_cols(const int64_t* rp, int n, int* col, double* val, int W, int far_den, uint64_t seed) {
+    int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    int64_t b = rp[i];
+    int len = (int)(rp[i + 1] - b);
+    int c[32];
+    for (int k = 0; k < len; ++k) {
+        uint64_t h = mix(seed ^ ((uint64_t)i * 0x9E3779B97F4A7C15ull) ^ ((uint64_t)(k + 1) * 0xBF58476D1CE4E5B9ull));
+        uint64_t h2 = mix(h);
+        int cc;
+        if ((int)(h % far_den) == 0) {
+            cc = (int)((h2 & 0xffffffffull) * (uint64_t)n >> 32);
+        } else {
+            int lo = max(0, i - W), hi = min(n - 1, i + W);
+            cc = lo + (int)((h2 & 0xffffffffull) * (uint64_t)(hi - lo + 1) >> 32);
+        }
+        c[k] = cc;
+        val[b + k] = (double)(int64_t)(h2 >> 40) * 0x1p-23 - 1.0;
+    }
+    for (int a = 1; a < len; ++a)
+        for (int q = a; q > 0 && c[q - 1] > c[q]; --q) {
+            int t = c[q];
+            c[q] = c[q - 1];
+            c[q - 1] = t;
+        }
+    for (int k = 0; k < len; ++k) col[b + k] = c[k];
+}
+
+__device__ cudaTextureObject_t g_xtex;
+
+// XM: 0 ldg, 1 tex, 2 mix (odd entries tex), 3 no gather, 4 ld.global (no .nc), 5 ld.global.nc.L1::evict_last
+template <int XM>
+__device__ __forceinline__ double ldx(const double* x, int c, int q) {
+    if constexpr (XM == 0) {
+        return __ldg(x + c);
+    } else if constexpr (XM == 1) {
+        const int2 t = tex1Dfetch<int2>(g_xtex, c);
+        return __hiloint2double(t.y, t.x);
+    } else if constexpr (XM == 2) {
+        if (q & 1) {
+            const int2 t = tex1Dfetch<int2>(g_xtex, c);
+            return __hiloint2double(t.y, t.x);
+        }
+        return __ldg(x + c);
+    } else if constexpr (XM == 3) {
+        return (double)c;
+    } else if constexpr (XM == 4) {
+        double r;
+        asm volatile("ld.global.f64 %0, [%1];" : "=d"(r) : "l"(x + c));
+        return r;
+    } else if constexpr (XM == 5) {
+        double r;
+        asm volatile("ld.global.nc.L1::evict_last.f64 %0, [%1];" : "=d"(r) : "l"(x + c));
+        return r;
+    } else if constexpr (XM == 6) {
+        double r;
+        asm volatile("ld.global.nc.L1::evict_first.f64 %0, [%1];" : "=d"(r) : "l"(x + c));
+        return r;
+    } else {
+        uint64_t pl;
+        asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pl));
+        double r;
+        asm volatile("ld.global.nc.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(r) : "l"(x + c), "l"(pl));
+        return r;
+    }
+}
+
+// the headline's structure: blocked teams, group of S lanes per row, quad tuples
+// (int4 colind + one 256-bit val load), lane l takes tuples l, l+S, ...
+// PC (CSR tuple loads): 0 __ldg, 1 L2::evict_first, 2 L1::evict_last + L2::evict_first,
+// 3 L1::no_allocate + L2::evict_first, 4 L2::evict_first on half the lines (fractional 0.5)
+template <int PC>
+__device__ __forceinline__ void ld_quad(const int* col, const double* val, uint64_t pol, int (&c)[4], double (&v)[4]) {
+    if constexpr (PC == 0) {
+        const int4 cc = __ldg(reinterpret_cast<const int4*>(col));
+        c[0] = cc.x, c[1] = cc.y, c[2] = cc.z, c[3] = cc.w;
+        asm("ld.global.nc.v4.f64 {%0, %1, %2, %3}, [%4];" : "=d"(v[0]), "=d"(v[1]), "=d"(v[2]), "=d"(v[3]) : "l"(val));
+    } else if constexpr (PC == 1 || PC == 4) {
+        asm("ld.global.nc.L2::cache_hint.v4.s32 {%0, %1, %2, %3}, [%4], %5;"
+            : "=r"(c[0]), "=r"(c[1]), "=r"(c[2]), "=r"(c[3]) : "l"(col), "l"(pol));
+        asm("ld.global.nc.L2::cache_hint.v4.f64 {%0, %1, %2, %3}, [%4], %5;"
+            : "=d"(v[0]), "=d"(v[1]), "=d"(v[2]), "=d"(v[3]) : "l"(val), "l"(pol));
+    } else if constexpr (PC == 2) {
+        asm("ld.global.nc.L1::evict_last.L2::cache_hint.v4.s32 {%0, %1, %2, %3}, [%4], %5;"
+            : "=r"(c[0]), "=r"(c[1]), "=r"(c[2]), "=r"(c[3]) : "l"(col), "l"(pol));
+        asm("ld.global.nc.L1::evict_last.L2::cache_hint.v4.f64 {%0, %1, %2, %3}, [%4], %5;"
+            : "=d"(v[0]), "=d"(v[1]), "=d"(v[2]), "=d"(v[3]) : "l"(val), "l"(pol));
+    } else {
+        asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.s32 {%0, %1, %2, %3}, [%4], %5;"
+            : "=r"(c[0]), "=r"(c[1]), "=r"(c[2]), "=r"(c[3]) : "l"(col), "l"(pol));
+        asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.f64 {%0, %1, %2, %3}, [%4], %5;"
+            : "=d"(v[0]), "=d"(v[1]), "=d"(v[2]), "=d"(v[3]) : "l"(val), "l"(pol));
+    }
+}
+
+template <int S, int XM, int PC = 0>
+__global__ void __launch_bounds__(1024, 2)
+    spmv_q(const int64_t* __restrict__ rp, const int* __restrict__ col, const double* __restrict__ val,
+           const double* __restrict__ x, double* __restrict__ y, int n, int chunk, int nnz) {
+    const int G = blockDim.x / S;
+    const int g = threadIdx.x / S, lane = threadIdx.x % S;
+    const int cs = blockIdx.x * chunk;
+    const int ce = min(n, cs + chunk);
+    uint64_t pol = 0;
+    if constexpr (PC == 4) {
+        asm("createpolicy.fractional.L2::evict_first.L2::evict_unchanged.b64 %0, 0.5;" : "=l"(pol));
+    } else if constexpr (PC != 0) {
+        asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    }
+    for (int i = cs + g; i < ce; i += G) {
+        const int b = (int)__ldg(rp + i), e = (int)__ldg(rp + i + 1);
+        const int trip = e > b ? ((e + 3) >> 2) - (b >> 2) : 0;
+        double acc = 0.0;
+        for (int t = lane; t < trip; t += S) {
+            const int k0 = ((b >> 2) + t) << 2;
+            int c[4];
+            double v[4];
+            if (k0 + 4 <= nnz) {
+                ld_quad<PC>(col + k0, val + k0, pol, c, v);
+            } else {
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    const int kq = k0 + q < nnz ? k0 + q : k0;
+                    c[q] = __ldg(col + kq);
+                    v[q] = __ldg(val + kq);
+                }
+            }
+#pragma unroll
+            for (int q = 0; q < 4; ++q)
+                if (k0 + q >= b && k0 + q < e) acc = fma(v[q], ldx<XM>(x, c[q], q), acc);
+        }
+#pragma unroll
+        for (int off = S / 2; off >= 1; off >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, off);
+        if (lane == 0) y[i] = acc;
+    }
+}
+
+// Diagnostic for the DRAM side: the same nonzeros and gathers as the SpMV, but the
+// CSR stream read in full lines (warp-coalesced, lane = nonzero) with a chosen L2
+// policy, the x gathers with another; one sum per thread (no rows).  Does L2 keep
+// x (80-100 MB) while 1-1.3 GB of CSR streams through it?  ncu dram__bytes tells.
+// PC: 0 normal, 1 L2::evict_first, 2 L1::no_allocate + L2::evict_first
+// PX: 0 normal, 1 L2::evict_last
+template <int PC, int PX>
+__global__ void __launch_bounds__(1024, 2)
+    stream_gather(const int* __restrict__ col, const double* __restrict__ val, const double* __restrict__ x,
+                  int nnz, double* sink) {
+    uint64_t pf, pl;
+    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pf));
+    asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pl));
+    double acc = 0.0;
+    const int stride = gridDim.x * blockDim.x;
+    // blocked: each CTA sweeps a contiguous range (like the blocked teams)
+    const int per = (nnz + gridDim.x - 1) / gridDim.x;
+    const int b0 = blockIdx.x * per, e0 = min(nnz, b0 + per);
+    (void)stride;
+    for (int k = b0 + threadIdx.x; k < e0; k += blockDim.x) {
+        int c;
+        double v, xv;
+        if constexpr (PC == 0) {
+            c = __ldg(col + k), v = __ldg(val + k);
+        } else if constexpr (PC == 1) {
+            asm volatile("ld.global.nc.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(c) : "l"(col + k), "l"(pf));
+            asm volatile("ld.global.nc.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(v) : "l"(val + k), "l"(pf));
+        } else {
+            asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(c) : "l"(col + k), "l"(pf));
+            asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(v) : "l"(val + k), "l"(pf));
+        }
+        if constexpr (PX == 0) {
+            xv = __ldg(x + c);
+        } else {
+            asm volatile("ld.global.nc.L2::cache_hint.f64 %0, [%1], %2;" : "=d"(xv) : "l"(x + c), "l"(pl));
+        }
+        acc = fma(v, xv, acc);
+    }
+    if (acc == 1234.5) sink[0] = acc;
+}
+
+// ----------------------------------------------------------------------------
+// Warp-staged CSR (experiment): warp = 32/S groups = a batch of RB = 32/S
+// consecutive rows of the team's range.  The warp loads the batch's rowptr slice
+// (one coalesced load) and its whole colind/val range in 4-nonzero units with
+// full-line loads (POL 1: L1::no_allocate + L2::evict_first, so x stays in L2),
+// stores them to its shared stage, and each group runs its row's simd loop from
+// the stage: lane id takes nonzeros id, id+S, ... (Fig 8 order, scalar).  A batch
+// whose range exceeds the stage falls back to direct loads.
+template <int POL>
+__device__ __forceinline__ void ld_unit(const int* col, const double* val, uint64_t pol, int4& c, double (&v)[4]) {
+    if constexpr (POL == 0) {
+        c = __ldg(reinterpret_cast<const int4*>(col));
+        asm volatile("ld.global.nc.v4.f64 {%0, %1, %2, %3}, [%4];" : "=d"(v[0]), "=d"(v[1]), "=d"(v[2]), "=d"(v[3]) : "l"(val));
+    } else {
+        asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.s32 {%0, %1, %2, %3}, [%4], %5;"
+                     : "=r"(c.x), "=r"(c.y), "=r"(c.z), "=r"(c.w) : "l"(col), "l"(pol));
+        asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.f64 {%0, %1, %2, %3}, [%4], %5;"
+                     : "=d"(v[0]), "=d"(v[1]), "=d"(v[2]), "=d"(v[3]) : "l"(val), "l"(pol));
+    }
+}
+
+template <int S, int CAPU, int H, int TPB, int MINB, int POL, bool RPF>
+__global__ void __launch_bounds__(TPB, MINB)
+    spmv_ws(const int64_t* __restrict__ rp, const int* __restrict__ col, const double* __restrict__ val,
+            const double* __restrict__ x, double* __restrict__ y, int n, int chunk, int nnz) {
+    constexpr int RB = 32 / S;
+    extern __shared__ __align__(16) unsigned char sm_raw[];
+    const int W = TPB / 32, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    int* scol = reinterpret_cast<int*>(sm_raw) + w * CAPU * 4;
+    double* sval = reinterpret_cast<double*>(sm_raw + (size_t)W * CAPU * 16) + w * CAPU * 4;
+    uint64_t pol = 0;
+    if constexpr (POL == 1) asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    const int g = lane / S, id = lane % S;
+    const int cs = blockIdx.x * chunk;
+    const int ce = min(n, cs + chunk);
+    const int nb = (ce - cs + RB - 1) / RB;
+    int m = w;
+    long long rpn = 0;
+    if (RPF && m < nb) {
+        const int r = cs + m * RB + lane;
+        if (lane <= RB) rpn = __ldg(rp + min(r, ce));
+    }
+    for (; m < nb; m += W) {
+        const int r0 = cs + m * RB;
+        const int nr = min(RB, ce - r0);
+        long long rpl;
+        if constexpr (RPF) {
+            rpl = rpn;
+            const int r = cs + (m + W) * RB + lane;
+            if (m + W < nb && lane <= RB) rpn = __ldg(rp + min(r, ce));
+        } else {
+            rpl = lane <= RB ? __ldg(rp + min(r0 + lane, ce)) : 0;
+        }
+        const int kb = (int)__shfl_sync(0xffffffffu, rpl, 0);
+        const int ke = (int)__shfl_sync(0xffffffffu, rpl, nr);
+        const int b = (int)__shfl_sync(0xffffffffu, rpl, min(g, nr));
+        const int e = (int)__shfl_sync(0xffffffffu, rpl, min(g + 1, nr));
+        const int u0 = kb >> 2;
+        const int nu = ((ke + 3) >> 2) - u0;
+        double acc = 0.0;
+        if (nu <= CAPU) {
+            for (int u = lane; u < nu; u += 32) {
+                const int k0 = (u0 + u) << 2;
+                int4 c;
+                double v[4];
+                if (k0 + 4 <= nnz) {
+                    ld_unit<POL>(col + k0, val + k0, pol, c, v);
+                } else {
+                    c.x = __ldg(col + k0);
+                    c.y = k0 + 1 < nnz ? __ldg(col + k0 + 1) : 0;
+                    c.z = k0 + 2 < nnz ? __ldg(col + k0 + 2) : 0;
+                    c.w = k0 + 3 < nnz ? __ldg(col + k0 + 3) : 0;
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) v[q] = k0 + q < nnz ? __ldg(val + k0 + q) : 0.0;
+                }
+                reinterpret_cast<int4*>(scol)[u] = c;
+                reinterpret_cast<double2*>(sval)[2 * u] = make_double2(v[0], v[1]);
+                reinterpret_cast<double2*>(sval)[2 * u + 1] = make_double2(v[2], v[3]);
+            }
+            __syncwarp();
+            const int o = b - (u0 << 2);
+            const int len = e - b;
+            // head block of H iterations: smem loads, then gathers, then folds (Fig 8 order)
+            int cc[H];
+            double vv[H], xv[H];
+#pragma unroll
+            for (int h = 0; h < H; ++h) {
+                const int j = id + h * S;
+                cc[h] = j < len ? scol[o + j] : 0;
+                vv[h] = j < len ? sval[o + j] : 0.0;
+            }
+#pragma unroll
+            for (int h = 0; h < H; ++h) xv[h] = id + h * S < len ? __ldg(x + cc[h]) : 0.0;
+#pragma unroll
+            for (int h = 0; h < H; ++h)
+                if (id + h * S < len) acc = fma(vv[h], xv[h], acc);
+            for (int j = id + H * S; j < len; j += S) acc = fma(sval[o + j], __ldg(x + scol[o + j]), acc);
+            __syncwarp();
+        } else {
+            for (int j = id; j < e - b; j += S) acc = fma(__ldg(val + b + j), __ldg(x + __ldg(col + b + j)), acc);
+        }
+#pragma unroll
+        for (int off = S / 2; off >= 1; off >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, off);
+        if (id == 0 && g < nr) y[r0 + g] = acc;
+    }
+}
+
+// reference for the staged kernels' order: scalar Fig 8 (lane id: id, id+S, ...)
+template <int S>
+__global__ void __launch_bounds__(1024, 2)
+    spmv_s(const int64_t* __restrict__ rp, const int* __restrict__ col, const double* __restrict__ val,
+           const double* __restrict__ x, double* __restrict__ y, int n, int chunk, int nnz) {
+    const int G = blockDim.x / S;
+    const int g = threadIdx.x / S, id = threadIdx.x % S;
+    const int cs = blockIdx.x * chunk;
+    const int ce = min(n, cs + chunk);
+    for (int i = cs + g; i < ce; i += G) {
+        const int b = (int)__ldg(rp + i), e = (int)__ldg(rp + i + 1);
+        double acc = 0.0;
+        for (int j = id; j < e - b; j += S) acc = fma(__ldg(val + b + j), __ldg(x + __ldg(col + b + j)), acc);
+#pragma unroll
+        for (int off = S / 2; off >= 1; off >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, off);
+        if (id == 0) y[i] = acc;
+    }
+}
+
+__global__ void flush_kernel(int4* p, size_t n) {
+    for (size_t k = blockIdx.x * (size_t)blockDim.x + threadIdx.x; k < n; k += (size_t)gridDim.x * blockDim.x)
+        p[k] = make_int4((int)k, 1, 2, 3);
+}
+
+typedef void (*SpmvFn)(const int64_t*, const int*, const double*, const double*, double*, int, int, int);
+
+int main(int argc, char** argv) {
+    const int n = argc > 1 ? atoi(argv[1]) : 10000000;
+    const int far_den = argc > 2 ? atoi(argv[2]) : 16;
+    cudaDeviceProp prop;
+    CK(cudaGetDeviceProperties(&prop, 0));
+    const size_t flush_bytes = 512ull << 20;
+    int4* fl;
+    CK(cudaMalloc(&fl, flush_bytes));
+    cudaEvent_t e0, e1;
+    CK(cudaEventCreate(&e0));
+    CK(cudaEventCreate(&e1));
+    std::vector<int64_t> rp(n + 1);
+    rp[0] = 0;
+    for (int i = 0; i < n; ++i) rp[i + 1] = rp[i] + 4 + (int)(mix(20230809ull ^ (uint64_t)i * 77) % 9);
+    const int nnz = (int)rp[n];
+    int64_t* drp;
+    int* dcol;
+    double *dval, *dx, *dy, *dy0;
+    CK(cudaMalloc(&drp, (n + 1) * 8ull));
+    CK(cudaMalloc(&dcol, nnz * 4ull));
+    CK(cudaMalloc(&dval, nnz * 8ull + 64));
+    CK(cudaMalloc(&dx, n * 8ull));
+    CK(cudaMalloc(&dy, n * 8ull));
+    CK(cudaMalloc(&dy0, n * 8ull));
+    CK(cudaMemcpy(drp, rp.data(), (n + 1) * 8ull, cudaMemcpyHostToDevice));
+    gen_cols<<<(n + 255) / 256, 256>>>(drp, n, dcol, dval, 4096, far_den, 20230809ull);
+    std::vector<double> hx(n);
+    for (int i = 0; i < n; ++i) hx[i] = (double)(mix(i * 3ull + 1) >> 11) * 0x1p-53 * 2 - 1;
+    CK(cudaMemcpy(dx, hx.data(), n * 8ull, cudaMemcpyHostToDevice));
+    cudaResourceDesc rd;
+    memset(&rd, 0, sizeof(rd));
+    rd.resType = cudaResourceTypeLinear;
+    rd.res.linear.devPtr = dx;
+    rd.res.linear.desc = cudaCreateChannelDesc<int2>();
+    rd.res.linear.sizeInBytes = n * 8ull;
+    cudaTextureDesc td;
+    memset(&td, 0, sizeof(td));
+    td.readMode = cudaReadModeElementType;
+    cudaTextureObject_t tex;
+    CK(cudaCreateTextureObject(&tex, &rd, &td, nullptr));
+    CK(cudaMemcpyToSymbol(g_xtex, &tex, sizeof(tex)));
+    CK(cudaDeviceSynchronize());
+    const double alg = nnz * 12.0 + (n + 1) * 8.0 + n * 8.0 + n * 8.0;
+    printf("# %s n=%d nnz=%d far 1/%d alg %.3f GB maxTex1DLinear %d\n", prop.name, n, nnz, far_den, alg * 1e-9,
+           prop.maxTexture1DLinear);
+    struct V {
+        const char* name;
+        SpmvFn fn;
+        int T = 1024;
+        int smem = 0;
+        const char* ref = nullptr;
+        int apw = 0;   // 1: persisting L2 access-policy window over x (reset before every launch)
+    } vs[] = {
+        {"S2 quads ldg (headline)", spmv_q<2, 0>, 1024, 0, "q"},
+        {"S2 quads apw 16MB", spmv_q<2, 0>, 1024, 0, nullptr, 16},
+        {"S2 quads apw 32MB", spmv_q<2, 0>, 1024, 0, nullptr, 32},
+        {"S2 quads apw 48MB", spmv_q<2, 0>, 1024, 0, nullptr, 48},
+        {"S2 quads apw 64MB", spmv_q<2, 0>, 1024, 0, nullptr, 64},
+        {"S2 quads apw max", spmv_q<2, 0>, 1024, 0, nullptr, 1000},
+        {"S2 quads apw 48MB csr L1el+L2ef", spmv_q<2, 0, 2>, 1024, 0, nullptr, 48},
+        {"S4 scalar apw 48MB", spmv_s<4>, 1024, 0, nullptr, 48},
+        {"S2 quads csr L2ef", spmv_q<2, 0, 1>},
+        {"S2 quads csr L1el+L2ef", spmv_q<2, 0, 2>},
+        {"S2 quads csr L1na+L2ef", spmv_q<2, 0, 3>},
+        {"S2 quads csr L2ef half", spmv_q<2, 0, 4>},
+        {"S2 quads csr L1el+L2ef x L1ef", spmv_q<2, 6, 2>},
+        {"S2 quads csr L2ef x L2el", spmv_q<2, 7, 1>},
+        {"S2 quads csr L1el+L2ef x L2el", spmv_q<2, 7, 2>},
+        {"S2 quads x L1ef", spmv_q<2, 6, 0>},
+        {"S2 scalar (ref for ws)", spmv_s<2>, 1024, 0, "ws"},
+        {"ws S2 cap48 H2 T1024x2 evf", spmv_ws<2, 48, 2, 1024, 2, 1, false>, 1024, 32 * 48 * 48},
+        {"ws S2 cap48 H4 T1024x1 evf rpf", spmv_ws<2, 48, 4, 1024, 1, 1, true>, 1024, 32 * 48 * 48},
+        {"S4 scalar (ref)", spmv_s<4>, 1024, 0, "s4"},
+        {"ws S4 cap32 H2 T1024x2 evf rpf", spmv_ws<4, 32, 2, 1024, 2, 1, true>, 1024, 32 * 32 * 48},
+        {"diag S2 quads no gather", spmv_q<2, 3>},
+    };
+    int k = 0;
+    for (auto& v : vs) {
+        ++k;
+        int nb = 0;
+        if (v.smem > 48 * 1024) CK(cudaFuncSetAttribute(v.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, v.smem));
+        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, v.fn, v.T, v.smem));
+        const int grid = prop.multiProcessorCount * nb;
+        int chunk = (n + grid - 1) / grid;
+        chunk = (chunk + 31) / 32 * 32;
+        std::vector<float> ts;
+        cudaStream_t st = 0;
+        if (v.apw) {
+            CK(cudaStreamCreate(&st));
+            const size_t setaside = std::min((size_t)prop.persistingL2CacheMaxSize, (size_t)v.apw << 20);
+            CK(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, setaside));
+            cudaStreamAttrValue a;
+            memset(&a, 0, sizeof(a));
+            a.accessPolicyWindow.base_ptr = dx;
+            a.accessPolicyWindow.num_bytes = std::min((size_t)n * 8, (size_t)prop.accessPolicyMaxWindowSize);
+            a.accessPolicyWindow.hitRatio = std::min(1.0f, (float)setaside / (float)a.accessPolicyWindow.num_bytes);
+            a.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+            a.accessPolicyWindow.missProp = cudaAccessPropertyNormal;
+            CK(cudaStreamSetAttribute(st, cudaStreamAttributeAccessPolicyWindow, &a));
+            printf("   apw: setaside %zu MB window %zu MB hitRatio %.2f\n", setaside >> 20,
+                   (size_t)a.accessPolicyWindow.num_bytes >> 20, a.accessPolicyWindow.hitRatio);
+        }
+        for (int r = 0; r < 13; ++r) {
+            if (v.apw) CK(cudaCtxResetPersistingL2Cache());
+            flush_kernel<<<4 * prop.multiProcessorCount, 1024, 0, st>>>(fl, flush_bytes / 16);
+            CK(cudaEventRecord(e0, st));
+            v.fn<<<grid, v.T, v.smem, st>>>(drp, dcol, dval, dx, dy, n, chunk, nnz);
+            CK(cudaEventRecord(e1, st));
+            CK(cudaEventSynchronize(e1));
+            float ms;
+            CK(cudaEventElapsedTime(&ms, e0, e1));
+            if (r >= 3) ts.push_back(ms);
+        }
+        CK(cudaGetLastError());
+        if (v.apw) {
+            cudaStreamAttrValue a;
+            memset(&a, 0, sizeof(a));
+            CK(cudaStreamSetAttribute(st, cudaStreamAttributeAccessPolicyWindow, &a));
+            CK(cudaCtxResetPersistingL2Cache());
+            CK(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, 0));
+            CK(cudaStreamSynchronize(st));
+            CK(cudaStreamDestroy(st));
+        }
+        std::sort(ts.begin(), ts.end());
+        const float med = ts[ts.size() / 2];
+        const char* tag = "(ref)";
+        if (v.ref) {
+            CK(cudaMemcpy(dy0, dy, n * 8ull, cudaMemcpyDeviceToDevice));
+        } else {
+            std::vector<double> a(n), b(n);
+            CK(cudaMemcpy(a.data(), dy, n * 8ull, cudaMemcpyDeviceToHost));
+            CK(cudaMemcpy(b.data(), dy0, n * 8ull, cudaMemcpyDeviceToHost));
+            tag = memcmp(a.data(), b.data(), n * 8ull) ? "differs" : "bit-identical";
+        }
+        printf("%2d %-28s grid %4d median %.4f ms min %.4f  %.0f GB/s alg  %s\n", k, v.name, grid, med, ts[0],
+               alg / med * 1e-6, tag);
+    }
+    // ---- DRAM-side diagnostic (stream_gather); time here, bytes under ncu
+    typedef void (*SgFn)(const int*, const double*, const double*, int, double*);
+    struct W {
+        const char* name;
+        SgFn fn;
+    } ws[] = {{"sg csr normal, x normal", stream_gather<0, 0>},
+              {"sg csr evict_first, x normal", stream_gather<1, 0>},
+              {"sg csr evict_first, x evict_last", stream_gather<1, 1>},
+              {"sg csr L1na+evict_first, x evict_last", stream_gather<2, 1>},
+              {"sg csr normal, x evict_last", stream_gather<0, 1>}};
+    for (auto& w : ws) {
+        std::vector<float> ts;
+        for (int r = 0; r < 8; ++r) {
+            flush_kernel<<<4 * prop.multiProcessorCount, 1024>>>(fl, flush_bytes / 16);
+            CK(cudaEventRecord(e0));
+            w.fn<<<2 * prop.multiProcessorCount, 1024>>>(dcol, dval, dx, nnz, dy);
+            CK(cudaEventRecord(e1));
+            CK(cudaEventSynchronize(e1));
+            float ms;
+            CK(cudaEventElapsedTime(&ms, e0, e1));
+            if (r >= 3) ts.push_back(ms);
+        }
+        CK(cudaGetLastError());
+        std::sort(ts.begin(), ts.end());
+        printf("   %-40s median %.4f ms\n", w.name, ts[ts.size() / 2]);
+    }
+    return 0;
+}

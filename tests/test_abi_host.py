@@ -32,7 +32,7 @@ def test_every_header_symbol_is_exported_and_bound():
 
 
 def test_abi_version_and_status_strings():
-    assert N.nest_abi_version() == N.NEST_ABI_VERSION == 1
+    assert N.nest_abi_version() == N.NEST_ABI_VERSION == 2
     assert N.nest_status_str(0) == b"NEST_OK"
     assert N.nest_status_str(2) == b"NEST_ERR_UNSUPPORTED"
 
@@ -231,3 +231,23 @@ def test_spmv_plan_index_width_covers_the_cyclic_schedule():
     assert small["index_bits"] == 32
     big = P.spmv_plan(1000, 1000, 8000, simdlen=1, threads_per_team=1024, num_teams=3_000_000)
     assert big["index_bits"] == 64
+
+
+def test_x_l2_persist_flag_rules():
+    # NEST_F_X_L2_PERSIST: CSR SpMV only (nest_kernel variants); rejected before any device call
+    with pytest.raises(P.NestError) as e:
+        P.plan(1000, 24, x_l2_persist=True)
+    assert e.value.status == N.NEST_ERR_INVALID_ARG and "SpMV" in str(e.value)
+    d = P.make_desc(x_l2_persist=True)
+    assert N.nest_batched_matvec_f32(ctypes.byref(d), 1, 64, 64, None, None, None, None) == N.NEST_ERR_INVALID_ARG
+    assert N.nest_nested_stencil_f64(ctypes.byref(d), 1, 4, None, None, None, None, None, None) == \
+        N.NEST_ERR_INVALID_ARG
+    with pytest.raises(P.NestError) as e:   # the x ring: unsupported
+        P.spmv_plan(1000, 1000, 8000, simdlen=2, x_halo=64, threads_per_team=256, x_l2_persist=True)
+    assert e.value.status == N.NEST_ERR_UNSUPPORTED and "x ring" in str(e.value)
+    with pytest.raises(P.NestError) as e:   # the two-level teams-generic baseline: unsupported
+        P.spmv_plan(1000, 1000, 8000, simdlen=1, mode="teams_generic", x_l2_persist=True)
+    assert e.value.status == N.NEST_ERR_UNSUPPORTED
+    assert N.NEST_F_X_L2_PERSIST == 1 << 6
+    with open(os.path.join(ROOT, "include", "nest.h")) as f:
+        assert "NEST_F_X_L2_PERSIST = 1u << 6" in f.read()

@@ -649,3 +649,52 @@ def test_laplace3d_vec128_rejects_odd_nx(P):
     u = R.laplace_inputs(4, 4, 5)
     with pytest.raises(Exception, match="even nx"):
         P.laplace3d_f64(dev(u), dev(u.copy()), 4, 4, 5, 0.125, vec128=True)
+
+
+# ------------------------------------------------------------------ a8 SpMV, x persisting in L2
+@pytest.mark.parametrize("S", (1, 2, 8))
+def test_spmv_x_l2_persist_is_a_cache_policy_only(P, banded, cfg1, S):
+    # NEST_F_X_L2_PERSIST changes where x lives in L2, never a result: bit-identical to the
+    # same launch without it, and to the oracle (integer data) / within R3 (real data)
+    for data in (banded, cfg1):
+        for values in ("int", "real"):
+            rp, col, val, x, yref, aref = data[values]
+            t = [dev(rp), dev(col), dev(val), dev(x)]
+            for cfg in (dict(), dict(blocked=True, threads_per_team=1024, vec128=True, quad=True),
+                        dict(blocked=True, vec128=True, mode="generic_smem"), dict(outer_unroll=2, mode="generic_shfl")):
+                y0 = host(P.spmv_csr_f64(*t, simdlen=S, **cfg))
+                y1 = host(P.spmv_csr_f64(*t, simdlen=S, x_l2_persist=True, **cfg))
+                assert np.array_equal(bits(y1), bits(y0)), cfg
+                if values == "int":
+                    assert np.array_equal(bits(y1), bits(yref)), cfg
+                else:
+                    assert_close(y1, yref, aref, 1e-12)
+
+
+def test_spmv_x_l2_persist_plan_and_flush(P, banded):
+    rp, col, val, x, yref, aref = banded["real"]
+    n = rp.size - 1
+    info = P.spmv_plan(n, x.size, val.size, simdlen=2, blocked=True, threads_per_team=1024, vec128=True, quad=True,
+                       x_l2_persist=True)
+    props = torch.cuda.get_device_properties(0)
+    assert info["l2_window_bytes"] == x.size * 8           # x (400 KB) is under the window whole
+    assert 0 < info["l2_setaside_bytes"] <= props.L2_cache_size
+    plain = P.spmv_plan(n, x.size, val.size, simdlen=2)
+    assert plain["l2_window_bytes"] == 0 and plain["l2_setaside_bytes"] == 0
+    # the flush utility returns persisting lines to normal and still flushes
+    t = [dev(rp), dev(col), dev(val), dev(x)]
+    buf = torch.empty(64 << 20, dtype=torch.uint8, device="cuda")
+    for _ in range(3):
+        y = P.spmv_csr_f64(*t, simdlen=2, blocked=True, threads_per_team=1024, vec128=True, quad=True,
+                           x_l2_persist=True)
+        P.l2_flush(buf)
+    torch.cuda.synchronize()
+    assert_close(host(y), yref, aref, 1e-12)
+    # the hostio (end-to-end) call takes the flag too: bit-identical to the device call
+    h = [torch.from_numpy(a).pin_memory() for a in (rp, col, val, x)]
+    h_y = torch.empty(n, dtype=torch.float64).pin_memory()
+    ws = torch.empty(P.hostio_workspace_bytes(n, x.size, val.size), dtype=torch.uint8, device="cuda")
+    P.spmv_csr_f64_hostio(*h, h_y, ws, simdlen=2, blocked=True, threads_per_team=1024, vec128=True, quad=True,
+                          x_l2_persist=True)
+    torch.cuda.synchronize()
+    assert np.array_equal(bits(h_y.numpy()), bits(host(y)))
