@@ -81,7 +81,7 @@ class ClockSampler:
     """nvidia-smi-equivalent clock / throttle sampling through NVML, run during
     the timed region."""
 
-    def __init__(self, index: int, period: float = 0.002):
+    def __init__(self, index: int, period: float = 0.001):
         self.samples, self.reasons = [], set()
         self.max_mhz = None
         self._stop = threading.Event()
@@ -117,13 +117,27 @@ class ClockSampler:
                     pass
             time.sleep(self._period)
 
+    def _sample_once(self):
+        nv = self._nv
+        if nv is not None:
+            try:
+                self.samples.append(nv.nvmlDeviceGetClockInfo(self._h, nv.NVML_CLOCK_SM))
+            except Exception:
+                pass
+
     def __enter__(self):
+        # short thread switch interval so the sampler runs while the main thread
+        # enqueues steps (the timed region is tens of ms); one sample on each edge
+        self._switch = sys.getswitchinterval()
+        sys.setswitchinterval(2e-4)
         self._t.start()
         return self
 
     def __exit__(self, *a):
+        self._sample_once()
         self._stop.set()
         self._t.join()
+        sys.setswitchinterval(self._switch)
 
     def summary(self):
         return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
