@@ -52,6 +52,12 @@ CONFIGS = {
                 dict(simdlen=S, vec128=v, team_chunk=c, **base))
                for S, v in ((8, True), (4, True), (2, True), (1, True), (8, False))
                for c in (0, 512, 2048, 8192, 32768)],
+    "xpol": [("S8 pairs", dict(simdlen=8, vec128=True, **base)),
+             ("S8 pairs persist", dict(simdlen=8, vec128=True, x_l2_persist=True, **base)),
+             ("S2 quads", dict(simdlen=2, quad=True, **base)),
+             ("S2 quads persist", dict(simdlen=2, quad=True, x_l2_persist=True, **base)),
+             ("S4 quads", dict(simdlen=4, quad=True, **base)),
+             ("S1 pairs", dict(simdlen=1, vec128=True, **base))],
     "hint": [("S8 pairs", dict(simdlen=8, vec128=True, **base)), ("S2 pairs", dict(simdlen=2, vec128=True, **base)),
              ("S4 pairs", dict(simdlen=4, vec128=True, **base)), ("S1 pairs", dict(simdlen=1, vec128=True, **base))],
     "unroll": [(f"S{S} {'pairs' if v else 'scalar'} U{U} T{T}", dict(simdlen=S, vec128=v, outer_unroll=U,

@@ -112,6 +112,15 @@ __device__ __forceinline__ void ld_quad(const int* col, const double* val, uint6
         const int4 cc = __ldg(reinterpret_cast<const int4*>(col));
         c[0] = cc.x, c[1] = cc.y, c[2] = cc.z, c[3] = cc.w;
         asm("ld.global.nc.v4.f64 {%0, %1, %2, %3}, [%4];" : "=d"(v[0]), "=d"(v[1]), "=d"(v[2]), "=d"(v[3]) : "l"(val));
+    } else if constexpr (PC == 5) {   // colind evict-first only
+        asm("ld.global.nc.L2::cache_hint.v4.s32 {%0, %1, %2, %3}, [%4], %5;"
+            : "=r"(c[0]), "=r"(c[1]), "=r"(c[2]), "=r"(c[3]) : "l"(col), "l"(pol));
+        asm("ld.global.nc.v4.f64 {%0, %1, %2, %3}, [%4];" : "=d"(v[0]), "=d"(v[1]), "=d"(v[2]), "=d"(v[3]) : "l"(val));
+    } else if constexpr (PC == 6) {   // val evict-first only
+        const int4 cc = __ldg(reinterpret_cast<const int4*>(col));
+        c[0] = cc.x, c[1] = cc.y, c[2] = cc.z, c[3] = cc.w;
+        asm("ld.global.nc.L2::cache_hint.v4.f64 {%0, %1, %2, %3}, [%4], %5;"
+            : "=d"(v[0]), "=d"(v[1]), "=d"(v[2]), "=d"(v[3]) : "l"(val), "l"(pol));
     } else if constexpr (PC == 1 || PC == 4) {
         asm("ld.global.nc.L2::cache_hint.v4.s32 {%0, %1, %2, %3}, [%4], %5;"
             : "=r"(c[0]), "=r"(c[1]), "=r"(c[2]), "=r"(c[3]) : "l"(col), "l"(pol));
@@ -400,27 +409,14 @@ int main(int argc, char** argv) {
         int apw = 0;   // 1: persisting L2 access-policy window over x (reset before every launch)
     } vs[] = {
         {"S2 quads ldg (headline)", spmv_q<2, 0>, 1024, 0, "q"},
-        {"S2 quads apw 16MB", spmv_q<2, 0>, 1024, 0, nullptr, 16},
-        {"S2 quads apw 32MB", spmv_q<2, 0>, 1024, 0, nullptr, 32},
-        {"S2 quads apw 48MB", spmv_q<2, 0>, 1024, 0, nullptr, 48},
-        {"S2 quads apw 64MB", spmv_q<2, 0>, 1024, 0, nullptr, 64},
-        {"S2 quads apw max", spmv_q<2, 0>, 1024, 0, nullptr, 1000},
-        {"S2 quads apw 48MB csr L1el+L2ef", spmv_q<2, 0, 2>, 1024, 0, nullptr, 48},
-        {"S4 scalar apw 48MB", spmv_s<4>, 1024, 0, nullptr, 48},
-        {"S2 quads csr L2ef", spmv_q<2, 0, 1>},
-        {"S2 quads csr L1el+L2ef", spmv_q<2, 0, 2>},
-        {"S2 quads csr L1na+L2ef", spmv_q<2, 0, 3>},
-        {"S2 quads csr L2ef half", spmv_q<2, 0, 4>},
-        {"S2 quads csr L1el+L2ef x L1ef", spmv_q<2, 6, 2>},
-        {"S2 quads csr L2ef x L2el", spmv_q<2, 7, 1>},
-        {"S2 quads csr L1el+L2ef x L2el", spmv_q<2, 7, 2>},
-        {"S2 quads x L1ef", spmv_q<2, 6, 0>},
-        {"S2 scalar (ref for ws)", spmv_s<2>, 1024, 0, "ws"},
-        {"ws S2 cap48 H2 T1024x2 evf", spmv_ws<2, 48, 2, 1024, 2, 1, false>, 1024, 32 * 48 * 48},
-        {"ws S2 cap48 H4 T1024x1 evf rpf", spmv_ws<2, 48, 4, 1024, 1, 1, true>, 1024, 32 * 48 * 48},
-        {"S4 scalar (ref)", spmv_s<4>, 1024, 0, "s4"},
-        {"ws S4 cap32 H2 T1024x2 evf rpf", spmv_ws<4, 32, 2, 1024, 2, 1, true>, 1024, 32 * 32 * 48},
-        {"diag S2 quads no gather", spmv_q<2, 3>},
+        {"S2 quads apw 63MB", spmv_q<2, 0>, 1024, 0, nullptr, 63},
+        {"S2 quads apw 63MB csr L2ef", spmv_q<2, 0, 1>, 1024, 0, nullptr, 63},
+        {"S2 quads apw 63MB col L2ef", spmv_q<2, 0, 5>, 1024, 0, nullptr, 63},
+        {"S2 quads apw 63MB val L2ef", spmv_q<2, 0, 6>, 1024, 0, nullptr, 63},
+        {"S2 quads apw 63MB csr L2ef half", spmv_q<2, 0, 4>, 1024, 0, nullptr, 63},
+        {"S2 quads apw 63MB csr L1el+L2ef", spmv_q<2, 0, 2>, 1024, 0, nullptr, 63},
+        {"S2 quads col L2ef", spmv_q<2, 0, 5>},
+        {"S2 quads val L2ef", spmv_q<2, 0, 6>},
     };
     int k = 0;
     for (auto& v : vs) {
