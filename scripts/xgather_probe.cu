@@ -139,10 +139,30 @@ __device__ __forceinline__ void ld_quad(const int* col, const double* val, uint6
     }
 }
 
-template <int S, int XM, int PC = 0>
+template <int S, int XM, int PC = 0, int PF = 0>
 __global__ void __launch_bounds__(1024, 2)
     spmv_q(const int64_t* __restrict__ rp, const int* __restrict__ col, const double* __restrict__ val,
            const double* __restrict__ x, double* __restrict__ y, int n, int chunk, int nnz) {
+    if constexpr (PF) {
+        // PF 1: the team's 1/grid share of x (far columns); PF 2: the team's own band
+        // [row0 - 4096, row1 + 4096); bulk L2 prefetches of <= 32 KB by warp 0
+        const int64_t xbytes = (int64_t)n * 8;
+        int64_t b0, e0;
+        if constexpr (PF == 1) {
+            const int64_t per = ((xbytes + gridDim.x - 1) / gridDim.x + 15) & ~(int64_t)15;
+            b0 = per * blockIdx.x, e0 = min(xbytes, b0 + per);
+        } else {
+            b0 = (int64_t)max(0, (int)blockIdx.x * chunk - 4096) * 8 & ~(int64_t)15;
+            e0 = min(xbytes, (int64_t)min(n, ((int)blockIdx.x + 1) * chunk + 4096) * 8);
+        }
+        if (threadIdx.x < 32)
+            for (int64_t o = b0 + (int64_t)threadIdx.x * 32768; o < e0; o += 32 * 32768) {
+                const uint32_t sz = (uint32_t)min((int64_t)32768, e0 - o) & ~15u;
+                if (sz)
+                    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(reinterpret_cast<const char*>(x) + o),
+                                 "r"(sz) : "memory");
+            }
+    }
     const int G = blockDim.x / S;
     const int g = threadIdx.x / S, lane = threadIdx.x % S;
     const int cs = blockIdx.x * chunk;
@@ -410,13 +430,11 @@ int main(int argc, char** argv) {
     } vs[] = {
         {"S2 quads ldg (headline)", spmv_q<2, 0>, 1024, 0, "q"},
         {"S2 quads apw 63MB", spmv_q<2, 0>, 1024, 0, nullptr, 63},
-        {"S2 quads apw 63MB csr L2ef", spmv_q<2, 0, 1>, 1024, 0, nullptr, 63},
-        {"S2 quads apw 63MB col L2ef", spmv_q<2, 0, 5>, 1024, 0, nullptr, 63},
-        {"S2 quads apw 63MB val L2ef", spmv_q<2, 0, 6>, 1024, 0, nullptr, 63},
-        {"S2 quads apw 63MB csr L2ef half", spmv_q<2, 0, 4>, 1024, 0, nullptr, 63},
-        {"S2 quads apw 63MB csr L1el+L2ef", spmv_q<2, 0, 2>, 1024, 0, nullptr, 63},
-        {"S2 quads col L2ef", spmv_q<2, 0, 5>},
-        {"S2 quads val L2ef", spmv_q<2, 0, 6>},
+        {"S2 quads apw 63MB + pf x share", spmv_q<2, 0, 0, 1>, 1024, 0, nullptr, 63},
+        {"S2 quads apw 63MB + pf band", spmv_q<2, 0, 0, 2>, 1024, 0, nullptr, 63},
+        {"S2 quads pf x share", spmv_q<2, 0, 0, 1>},
+        {"S2 quads pf band", spmv_q<2, 0, 0, 2>},
+        {"S2 quads apw 63MB", spmv_q<2, 0>, 1024, 0, nullptr, 63},
     };
     int k = 0;
     for (auto& v : vs) {
