@@ -247,6 +247,8 @@ CANDIDATES = [
     (2, "spmd", 1, 1024, 0, "bqp"),
     (2, "generic_smem", 1, 1024, 0, "b"),
     (2, "generic_shfl", 1, 1024, 0, "b"),
+    (2, "generic_smem", 1, 1024, 0, "bqp"),
+    (2, "generic_shfl", 1, 1024, 0, "bqp"),
     (4, "spmd", 1, 1024, 0, "bv"),
     (4, "spmd", 1, 1024, 0, "bq"),
     (4, "spmd", 1, 1024, 0, "bqp"),

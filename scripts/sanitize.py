@@ -29,6 +29,10 @@ for S in (2, 8, 32):
         P.nested_stencil_f64(inp, coef, w, 4099, 8, simdlen=S, mode=mode, outer_unroll=4)
         P.spmv_csr_f64(rp, col, val, x, simdlen=S, mode=mode, outer_unroll=2, threads_per_team=512)
         P.spmv_csr_f64(rp, col, val, x, simdlen=S, mode=mode, quad=True, blocked=True, threads_per_team=1024)
+        # x under a persisting-L2 access-policy window (cudaLaunchKernelEx), then the flush's reset
+        P.spmv_csr_f64(rp, col, val, x, simdlen=S, mode=mode, quad=True, blocked=True, threads_per_team=1024,
+                       x_l2_persist=True)
+        P.l2_flush(torch.empty(4 << 20, dtype=torch.uint8, device="cuda"))
         P.batched_matvec_f32(A, xb, 64, simdlen=S, mode=mode, outer_unroll=2)
         P.batched_matvec_f32(A, xb, 64, simdlen=S, mode=mode)   # lean SPMD / generic drivers (U = 1)
         P.spmv_csr_f64(rp, col, val, x, simdlen=S, mode=mode, blocked=True, vec128=True, threads_per_team=1024,
