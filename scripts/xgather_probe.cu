@@ -89,6 +89,10 @@ __device__ __forceinline__ double ldx(const double* x, int c, int q) {
         double r;
         asm volatile("ld.global.nc.L1::evict_last.f64 %0, [%1];" : "=d"(r) : "l"(x + c));
         return r;
+    } else if constexpr (XM == 8) {   // diagnostic: every gather an L1 hit (32 KB of x), distinct lines as before
+        return __ldg(x + (c & 4095));
+    } else if constexpr (XM == 9) {   // diagnostic: every gather an L1 hit, one line per 32 lanes (no line spread)
+        return __ldg(x + (c & 15));
     } else if constexpr (XM == 6) {
         double r;
         asm volatile("ld.global.nc.L1::evict_first.f64 %0, [%1];" : "=d"(r) : "l"(x + c));
@@ -368,6 +372,59 @@ __global__ void __launch_bounds__(1024, 2)
     }
 }
 
+// Co-located teams (diagnostic): the two teams resident on an SM sweep ONE region of
+// rows together (rounds of 2G consecutive rows, team slot s taking the s-th half), so
+// the SM's L1 holds one band of x instead of two.  Region = %smid; slot = parity of a
+// per-SM launch counter (exactly two teams per SM per launch: grid = 2 x SMs at an
+// occupancy of 2 -- checked by comparing y with the headline, bit for bit).
+__device__ int g_sm_ctr[256];
+template <int S>
+__global__ void __launch_bounds__(1024, 2)
+    spmv_colo(const int64_t* __restrict__ rp, const int* __restrict__ col, const double* __restrict__ val,
+              const double* __restrict__ x, double* __restrict__ y, int n, int chunk_unused, int nnz) {
+    __shared__ int s_slot, s_sm;
+    if (threadIdx.x == 0) {
+        int sm;
+        asm volatile("mov.u32 %0, %%smid;" : "=r"(sm));
+        s_sm = sm;
+        s_slot = atomicAdd(&g_sm_ctr[sm], 1) & 1;
+    }
+    __syncthreads();
+    const int nsm = gridDim.x / 2;
+    const int G = blockDim.x / S;
+    const int g = threadIdx.x / S, lane = threadIdx.x % S;
+    int per = (n + nsm - 1) / nsm;
+    per = (per + 2 * G - 1) / (2 * G) * (2 * G);
+    const int cs = s_sm * per;
+    const int ce = min(n, cs + per);
+    for (int i = cs + s_slot * G + g; i < ce; i += 2 * G) {
+        const int b = (int)__ldg(rp + i), e = (int)__ldg(rp + i + 1);
+        const int trip = e > b ? ((e + 3) >> 2) - (b >> 2) : 0;
+        double acc = 0.0;
+        for (int t = lane; t < trip; t += S) {
+            const int k0 = ((b >> 2) + t) << 2;
+            int c[4];
+            double v[4];
+            if (k0 + 4 <= nnz) {
+                ld_quad<0>(col + k0, val + k0, 0, c, v);
+            } else {
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    const int kq = k0 + q < nnz ? k0 + q : k0;
+                    c[q] = __ldg(col + kq);
+                    v[q] = __ldg(val + kq);
+                }
+            }
+#pragma unroll
+            for (int q = 0; q < 4; ++q)
+                if (k0 + q >= b && k0 + q < e) acc = fma(v[q], __ldg(x + c[q]), acc);
+        }
+#pragma unroll
+        for (int off = S / 2; off >= 1; off >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, off);
+        if (lane == 0) y[i] = acc;
+    }
+}
+
 __global__ void flush_kernel(int4* p, size_t n) {
     for (size_t k = blockIdx.x * (size_t)blockDim.x + threadIdx.x; k < n; k += (size_t)gridDim.x * blockDim.x)
         p[k] = make_int4((int)k, 1, 2, 3);
@@ -429,12 +486,9 @@ int main(int argc, char** argv) {
         int apw = 0;   // 1: persisting L2 access-policy window over x (reset before every launch)
     } vs[] = {
         {"S2 quads ldg (headline)", spmv_q<2, 0>, 1024, 0, "q"},
+        {"S2 quads co-located teams", spmv_colo<2>},
         {"S2 quads apw 63MB", spmv_q<2, 0>, 1024, 0, nullptr, 63},
-        {"S2 quads apw 63MB + pf x share", spmv_q<2, 0, 0, 1>, 1024, 0, nullptr, 63},
-        {"S2 quads apw 63MB + pf band", spmv_q<2, 0, 0, 2>, 1024, 0, nullptr, 63},
-        {"S2 quads pf x share", spmv_q<2, 0, 0, 1>},
-        {"S2 quads pf band", spmv_q<2, 0, 0, 2>},
-        {"S2 quads apw 63MB", spmv_q<2, 0>, 1024, 0, nullptr, 63},
+        {"S2 quads co-located apw 63MB", spmv_colo<2>, 1024, 0, nullptr, 63},
     };
     int k = 0;
     for (auto& v : vs) {
