@@ -52,6 +52,9 @@ CONFIGS = {
                 dict(simdlen=S, vec128=v, team_chunk=c, **base))
                for S, v in ((8, True), (4, True), (2, True), (1, True), (8, False))
                for c in (0, 512, 2048, 8192, 32768)],
+    "pshape": [(f"S{S} {'quads' if q else 'pairs'} T{T} persist", dict(simdlen=S, vec128=True, quad=q, blocked=True,
+                                                                      threads_per_team=T, x_l2_persist=True))
+               for S in (2, 4) for q in (True, False) for T in (512, 640, 768, 1024)],
     "xpol": [("S8 pairs", dict(simdlen=8, vec128=True, **base)),
              ("S8 pairs persist", dict(simdlen=8, vec128=True, x_l2_persist=True, **base)),
              ("S2 quads", dict(simdlen=2, quad=True, **base)),

@@ -116,6 +116,16 @@ __device__ __forceinline__ void ld_quad(const int* col, const double* val, uint6
         const int4 cc = __ldg(reinterpret_cast<const int4*>(col));
         c[0] = cc.x, c[1] = cc.y, c[2] = cc.z, c[3] = cc.w;
         asm("ld.global.nc.v4.f64 {%0, %1, %2, %3}, [%4];" : "=d"(v[0]), "=d"(v[1]), "=d"(v[2]), "=d"(v[3]) : "l"(val));
+    } else if constexpr (PC == 7) {   // L1::no_allocate only (L1 kept for the x band)
+        asm("ld.global.nc.L1::no_allocate.v4.s32 {%0, %1, %2, %3}, [%4];"
+            : "=r"(c[0]), "=r"(c[1]), "=r"(c[2]), "=r"(c[3]) : "l"(col));
+        asm("ld.global.nc.L1::no_allocate.v4.f64 {%0, %1, %2, %3}, [%4];"
+            : "=d"(v[0]), "=d"(v[1]), "=d"(v[2]), "=d"(v[3]) : "l"(val));
+    } else if constexpr (PC == 8) {   // val L1::no_allocate only
+        const int4 cc = __ldg(reinterpret_cast<const int4*>(col));
+        c[0] = cc.x, c[1] = cc.y, c[2] = cc.z, c[3] = cc.w;
+        asm("ld.global.nc.L1::no_allocate.v4.f64 {%0, %1, %2, %3}, [%4];"
+            : "=d"(v[0]), "=d"(v[1]), "=d"(v[2]), "=d"(v[3]) : "l"(val));
     } else if constexpr (PC == 5) {   // colind evict-first only
         asm("ld.global.nc.L2::cache_hint.v4.s32 {%0, %1, %2, %3}, [%4], %5;"
             : "=r"(c[0]), "=r"(c[1]), "=r"(c[2]), "=r"(c[3]) : "l"(col), "l"(pol));
@@ -486,9 +496,10 @@ int main(int argc, char** argv) {
         int apw = 0;   // 1: persisting L2 access-policy window over x (reset before every launch)
     } vs[] = {
         {"S2 quads ldg (headline)", spmv_q<2, 0>, 1024, 0, "q"},
-        {"S2 quads co-located teams", spmv_colo<2>},
         {"S2 quads apw 63MB", spmv_q<2, 0>, 1024, 0, nullptr, 63},
-        {"S2 quads co-located apw 63MB", spmv_colo<2>, 1024, 0, nullptr, 63},
+        {"S2 quads apw 63MB csr L1na", spmv_q<2, 0, 7>, 1024, 0, nullptr, 63},
+        {"S2 quads apw 63MB val L1na", spmv_q<2, 0, 8>, 1024, 0, nullptr, 63},
+        {"S2 quads csr L1na", spmv_q<2, 0, 7>},
     };
     int k = 0;
     for (auto& v : vs) {

@@ -41,6 +41,11 @@ def test_dist_spmv_single_rank_nccl():
             assert np.all(np.abs(y - yref) <= 1e-12 * aref)
             y1 = P.spmv_csr_f64(*d, simdlen=S, mode=mode, x_halo=halo).cpu().numpy()
             assert np.array_equal(y.view(np.int64), y1.view(np.int64))
+        # x_full under the persisting-L2 window: the same bits
+        y = comm.spmv_csr_f64(spec.nrows, spec.ncols, d[0], d[1], d[2], d[3], xf, simdlen=2, quad=True, blocked=True,
+                              threads_per_team=1024, x_l2_persist=True).cpu().numpy()
+        y1 = P.spmv_csr_f64(*d, simdlen=2, quad=True, blocked=True, threads_per_team=1024).cpu().numpy()
+        assert np.array_equal(y.view(np.int64), y1.view(np.int64))
         with pytest.raises(P.NestError):   # wrong local row count for the rank
             comm.spmv_csr_f64(spec.nrows + 5, spec.ncols, d[0], d[1], d[2], d[3], xf)
         # the exchange step alone, and the host-buffer entry point
@@ -51,7 +56,8 @@ def test_dist_spmv_single_rank_nccl():
         hy = torch.empty(spec.nrows, dtype=torch.float64).pin_memory()
         ws = torch.empty(comm.hostio_workspace_bytes(spec.nrows, val.size, spec.ncols), dtype=torch.uint8,
                          device="cuda")
-        for cfg in (dict(simdlen=2, quad=True, blocked=True, threads_per_team=1024), dict(simdlen=8)):
+        for cfg in (dict(simdlen=2, quad=True, blocked=True, threads_per_team=1024), dict(simdlen=8),
+                    dict(simdlen=2, quad=True, blocked=True, threads_per_team=1024, x_l2_persist=True)):
             comm.spmv_csr_f64_hostio(spec.nrows, spec.ncols, pin(rp), pin(col), pin(val), pin(x), hy, ws, **cfg)
             torch.cuda.synchronize()
             y1 = P.spmv_csr_f64(*d, **cfg).cpu().numpy()
