@@ -94,6 +94,9 @@ def test_xpeer_odd_chunks_and_errors(P):
             xp.spmv_csr_f64(spec.nrows + 50, *t)
         with pytest.raises(P.NestError):          # the x ring is not offered here
             xp.spmv_csr_f64(spec.nrows, *t, x_halo=100, threads_per_team=256)
+        with pytest.raises(P.NestError) as e:     # nor the persisting window (x is distributed)
+            xp.spmv_csr_f64(spec.nrows, *t, x_l2_persist=True)
+        assert e.value.status == P._nest.NEST_ERR_UNSUPPORTED
         xp.close()
 
 
