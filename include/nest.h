@@ -128,7 +128,8 @@ enum {
      * the caller's stream attributes are untouched.  Results are identical (a
      * cache policy only).  The persisting lines outlive the call (a following
      * SpMV on the same x finds them); nest_util_l2_flush returns them to
-     * normal.  With x_halo or NEST_MODE_TEAMS_GENERIC: NEST_ERR_UNSUPPORTED;
+     * normal, and nest_shutdown also restores the limit.  With x_halo,
+     * NEST_MODE_TEAMS_GENERIC or the peer-gather SpMV: NEST_ERR_UNSUPPORTED;
      * other entry points: NEST_ERR_INVALID_ARG. */
     NEST_F_X_L2_PERSIST = 1u << 6
 };
@@ -434,7 +435,9 @@ nest_status nest_spmv_csr_f64_xpeer(const nest_desc *desc, nest_xpeer *xp, int64
                                     void *stream);
 nest_status nest_xpeer_destroy(nest_xpeer *xp);
 
-/* Release library-owned device scratch of the current device. */
+/* Release library-owned device scratch of the current device; if a
+ * NEST_F_X_L2_PERSIST call raised the device's persisting-L2 limit, return the
+ * persisting lines to normal and restore the limit it found. */
 nest_status nest_shutdown(void);
 
 #ifdef __cplusplus

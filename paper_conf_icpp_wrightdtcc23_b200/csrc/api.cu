@@ -229,8 +229,8 @@ nest_status prepare_fallback(const Plan& p, unsigned char** fb, void* stream) {
 // 100 MB, profiles/r02s3_x_l2_persist.md): 63-71 MB beat 47 MB and the 79 MB
 // maximum (which leaves too little L2 for the streamed CSR lines).
 static std::mutex g_persist_mu;
-static std::map<int, int64_t> g_persist_set;   // device -> set-aside this library established
-static std::atomic<bool> g_persist_used{false};            // a persisting launch happened (nest_util_l2_flush resets)
+static std::map<int, size_t> g_persist_orig;       // device -> the limit before this library raised it
+static std::atomic<bool> g_persist_used{false};    // a persisting launch happened (nest_util_l2_flush resets)
 
 nest_status x_persist_window(Plan* p, const double* x, int64_t ncols, bool apply) {
     int dev = 0;
@@ -252,10 +252,10 @@ nest_status x_persist_window(Plan* p, const double* x, int64_t ncols, bool apply
     if (!apply) return NEST_OK;
     if ((int64_t)cur < want) {
         std::lock_guard<std::mutex> lk(g_persist_mu);
+        g_persist_orig.emplace(dev, cur);   // first raise only: nest_shutdown restores it
         if ((e = cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)want)) != cudaSuccess ||
             (e = cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize)) != cudaSuccess)   // granularity
             return cuda_fail(e, "cudaDeviceSetLimit(persisting L2)");
-        g_persist_set[dev] = (int64_t)cur;
         p->l2_setaside = (int64_t)cur;
     }
     g_persist_used = true;
@@ -753,6 +753,15 @@ NEST_API nest_status nest_shutdown(void) {
     if (h != g_hostio.end()) {
         hostio_destroy(h->second);
         g_hostio.erase(h);
+    }
+    // NEST_F_X_L2_PERSIST: persisting lines back to normal, the set-aside back to what it was
+    std::lock_guard<std::mutex> lk3(g_persist_mu);
+    auto q = g_persist_orig.find(dev);
+    if (q != g_persist_orig.end()) {
+        if ((e = cudaCtxResetPersistingL2Cache()) != cudaSuccess ||
+            (e = cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, q->second)) != cudaSuccess)
+            return cuda_fail(e, "restore the persisting-L2 limit");
+        g_persist_orig.erase(q);
     }
     return NEST_OK;
 }
