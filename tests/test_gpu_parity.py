@@ -698,3 +698,10 @@ def test_spmv_x_l2_persist_plan_and_flush(P, banded):
                           x_l2_persist=True)
     torch.cuda.synchronize()
     assert np.array_equal(bits(h_y.numpy()), bits(host(y)))
+    # nest_shutdown restores the persisting-L2 limit the library raised (0 on a fresh context)
+    from cuda.bindings import runtime as rt
+    lim = lambda: rt.cudaDeviceGetLimit(rt.cudaLimit.cudaLimitPersistingL2CacheSize)[1]
+    during = lim()
+    assert during >= info["l2_setaside_bytes"] > 0
+    P.shutdown()
+    assert lim() < during
