@@ -1,5 +1,5 @@
 """NEST_F_X_L2_PERSIST set-aside sweep (developer tool): the library raises the
-device's persisting-L2 limit to 3/8 of L2 and uses max(limit, that); here the
+device's persisting-L2 limit to half of L2 and uses max(limit, that); here the
 limit is raised further by hand and the headline quads timed on cfg2 and G100
 (median of 10 launches, L2 flushed and persisting lines reset before each)."""
 import os
