@@ -435,6 +435,88 @@ __global__ void __launch_bounds__(1024, 2)
     }
 }
 
+// ----------------------------------------------------------------------------
+// Static x window per team (experiment): non-persistent grid, team = C consecutive
+// rows; thread 0 bulk-copies x[lo, hi) = [r0 - H, r0 + C + H) (clipped, 16-byte
+// aligned) into shared memory at team start on one mbarrier; every warp loads its
+// first row's bounds and tuples BEFORE waiting on it (the copy hides behind the CSR
+// latency).  Gathers inside the window read shared memory, the rest global memory.
+__device__ __forceinline__ uint32_t sptr(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+template <int S, int C, int H>
+__global__ void __launch_bounds__(1024, 2)
+    spmv_win(const int64_t* __restrict__ rp, const int* __restrict__ col, const double* __restrict__ val,
+             const double* __restrict__ x, double* __restrict__ y, int n, int chunk_unused, int nnz) {
+    extern __shared__ __align__(16) double win[];
+    __shared__ __align__(8) uint64_t bar;
+    const int r0 = blockIdx.x * C;
+    const int r1 = min(n, r0 + C);
+    const int lo = max(0, r0 - H) & ~1;
+    const int hi = min(n, ((r1 + H) + 1) & ~1);   // n even in these matrices
+    const uint32_t bytes = (uint32_t)(hi - lo) * 8u;
+    if (threadIdx.x == 0) {
+        asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(sptr(&bar)));
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(sptr(&bar)), "r"(bytes) : "memory");
+        for (uint32_t o = 0; o < bytes; o += 16384) {
+            const uint32_t sz = min(16384u, bytes - o);
+            asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                         ::"r"(sptr(win) + o), "l"(reinterpret_cast<const char*>(x + lo) + o), "r"(sz), "r"(sptr(&bar))
+                         : "memory");
+        }
+    }
+    const int G = blockDim.x / S;
+    const int g = threadIdx.x / S, lane = threadIdx.x % S;
+    const unsigned wlen = (unsigned)(hi - lo);
+    bool waited = false;
+    for (int i = r0 + g; i < r1; i += G) {
+        const int b = (int)__ldg(rp + i), e = (int)__ldg(rp + i + 1);
+        const int trip = e > b ? ((e + 3) >> 2) - (b >> 2) : 0;
+        double acc = 0.0;
+        for (int t = lane; t < trip; t += S) {
+            const int k0 = ((b >> 2) + t) << 2;
+            int c[4];
+            double v[4];
+            if (k0 + 4 <= nnz) {
+                ld_quad<0>(col + k0, val + k0, 0, c, v);
+            } else {
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    const int kq = k0 + q < nnz ? k0 + q : k0;
+                    c[q] = __ldg(col + kq);
+                    v[q] = __ldg(val + kq);
+                }
+            }
+            if (!waited) {
+                asm volatile("{\n .reg .pred p;\n W: mbarrier.try_wait.parity.shared::cta.b64 p, [%0], 0;\n @!p bra W;\n}"
+                             ::"r"(sptr(&bar)) : "memory");
+                waited = true;
+            }
+            double xv[4];
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {   // branch-free: one predicated shared and one predicated global load
+                const unsigned off = (unsigned)(c[q] - lo);
+                const uint32_t sa = sptr(win) + (off < wlen ? off : 0u) * 8u;
+                asm volatile("{\n .reg .pred p;\n setp.lt.u32 p, %1, %2;\n @p ld.shared.f64 %0, [%3];\n"
+                             " @!p ld.global.nc.f64 %0, [%4];\n}"
+                             : "=d"(xv[q]) : "r"(off), "r"(wlen), "r"(sa), "l"(x + c[q]));
+            }
+#pragma unroll
+            for (int q = 0; q < 4; ++q)
+                if (k0 + q >= b && k0 + q < e) acc = fma(v[q], xv[q], acc);
+        }
+#pragma unroll
+        for (int off = S / 2; off >= 1; off >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, off);
+        if (lane == 0) y[i] = acc;
+    }
+    if (!waited)   // never leave a bulk copy in flight into a released shared-memory block
+        asm volatile("{\n .reg .pred p;\n W2: mbarrier.try_wait.parity.shared::cta.b64 p, [%0], 0;\n @!p bra W2;\n}"
+                     ::"r"(sptr(&bar)) : "memory");
+}
+
 __global__ void flush_kernel(int4* p, size_t n) {
     for (size_t k = blockIdx.x * (size_t)blockDim.x + threadIdx.x; k < n; k += (size_t)gridDim.x * blockDim.x)
         p[k] = make_int4((int)k, 1, 2, 3);
@@ -493,13 +575,19 @@ int main(int argc, char** argv) {
         int T = 1024;
         int smem = 0;
         const char* ref = nullptr;
-        int apw = 0;   // 1: persisting L2 access-policy window over x (reset before every launch)
+        int apw = 0;   // set-aside MB of a persisting L2 access-policy window over x (reset before every launch)
+        int rows_per_team = 0;   // > 0: non-persistent grid of ceil(n / rows_per_team) teams
     } vs[] = {
         {"S2 quads ldg (headline)", spmv_q<2, 0>, 1024, 0, "q"},
         {"S2 quads apw 63MB", spmv_q<2, 0>, 1024, 0, nullptr, 63},
-        {"S2 quads apw 63MB csr L1na", spmv_q<2, 0, 7>, 1024, 0, nullptr, 63},
-        {"S2 quads apw 63MB val L1na", spmv_q<2, 0, 8>, 1024, 0, nullptr, 63},
-        {"S2 quads csr L1na", spmv_q<2, 0, 7>},
+        {"win C2048 H2048", spmv_win<2, 2048, 2048>, 1024, (2048 + 4096 + 2) * 8, nullptr, 0, 2048},
+        {"win C4096 H2048", spmv_win<2, 4096, 2048>, 1024, (4096 + 4096 + 2) * 8, nullptr, 0, 4096},
+        {"win C2048 H4096", spmv_win<2, 2048, 4096>, 1024, (2048 + 8192 + 2) * 8, nullptr, 0, 2048},
+        {"win C4096 H4096", spmv_win<2, 4096, 4096>, 1024, (4096 + 8192 + 2) * 8, nullptr, 0, 4096},
+        {"win C8192 H2048", spmv_win<2, 8192, 2048>, 1024, (8192 + 4096 + 2) * 8, nullptr, 0, 8192},
+        {"win C4096 H2048 apw", spmv_win<2, 4096, 2048>, 1024, (4096 + 4096 + 2) * 8, nullptr, 63, 4096},
+        {"win C2048 H4096 apw", spmv_win<2, 2048, 4096>, 1024, (2048 + 8192 + 2) * 8, nullptr, 63, 2048},
+        {"win C4096 H4096 apw", spmv_win<2, 4096, 4096>, 1024, (4096 + 8192 + 2) * 8, nullptr, 63, 4096},
     };
     int k = 0;
     for (auto& v : vs) {
@@ -507,7 +595,7 @@ int main(int argc, char** argv) {
         int nb = 0;
         if (v.smem > 48 * 1024) CK(cudaFuncSetAttribute(v.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, v.smem));
         CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, v.fn, v.T, v.smem));
-        const int grid = prop.multiProcessorCount * nb;
+        const int grid = v.rows_per_team ? (n + v.rows_per_team - 1) / v.rows_per_team : prop.multiProcessorCount * nb;
         int chunk = (n + grid - 1) / grid;
         chunk = (chunk + 31) / 32 * 32;
         std::vector<float> ts;
