@@ -55,6 +55,10 @@ CONFIGS = {
     "pshape": [(f"S{S} {'quads' if q else 'pairs'} T{T} persist", dict(simdlen=S, vec128=True, quad=q, blocked=True,
                                                                       threads_per_team=T, x_l2_persist=True))
                for S in (2, 4) for q in (True, False) for T in (512, 640, 768, 1024)],
+    "cfg5": [(f"S{S} {'quads' if q else 'pairs'} U{U}{' persist' if pe else ''}",
+              dict(simdlen=S, vec128=True, quad=q, blocked=True, threads_per_team=1024, outer_unroll=U,
+                   x_l2_persist=pe))
+             for S in (4, 8, 16) for q in (True, False) for U in (1, 2) for pe in (False, True)],
     "xpol": [("S8 pairs", dict(simdlen=8, vec128=True, **base)),
              ("S8 pairs persist", dict(simdlen=8, vec128=True, x_l2_persist=True, **base)),
              ("S2 quads", dict(simdlen=2, quad=True, **base)),
