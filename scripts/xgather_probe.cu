@@ -517,6 +517,77 @@ __global__ void __launch_bounds__(1024, 2)
                      ::"r"(sptr(&bar)) : "memory");
 }
 
+// Head block of H quads per lane (all tuple loads, then all gathers, then the folds in
+// order), then the plain loop; launch bounds (TB, MINB) set the register budget.
+template <int S, int H, int TB, int MINB>
+__global__ void __launch_bounds__(TB, MINB)
+    spmv_qh(const int64_t* __restrict__ rp, const int* __restrict__ col, const double* __restrict__ val,
+            const double* __restrict__ x, double* __restrict__ y, int n, int chunk, int nnz) {
+    const int G = blockDim.x / S;
+    const int g = threadIdx.x / S, lane = threadIdx.x % S;
+    const int cs = blockIdx.x * chunk;
+    const int ce = min(n, cs + chunk);
+    for (int i = cs + g; i < ce; i += G) {
+        const int b = (int)__ldg(rp + i), e = (int)__ldg(rp + i + 1);
+        const int trip = e > b ? ((e + 3) >> 2) - (b >> 2) : 0;
+        double acc = 0.0;
+        int c[H][4];
+        double v[H][4];
+#pragma unroll
+        for (int h = 0; h < H; ++h) {
+            const int t = lane + h * S;
+            const int k0 = ((b >> 2) + t) << 2;
+            if (t < trip && k0 + 4 <= nnz) {
+                ld_quad<0>(col + k0, val + k0, 0, c[h], v[h]);
+            } else {
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    const int kq = min(k0 + q, nnz - 1);
+                    c[h][q] = t < trip ? __ldg(col + kq) : 0;
+                    v[h][q] = t < trip ? __ldg(val + kq) : 0.0;
+                }
+            }
+        }
+        double xv[H][4];
+#pragma unroll
+        for (int h = 0; h < H; ++h) {
+            const int t = lane + h * S;
+            const int k0 = ((b >> 2) + t) << 2;
+#pragma unroll
+            for (int q = 0; q < 4; ++q) xv[h][q] = (t < trip && k0 + q >= b && k0 + q < e) ? __ldg(x + c[h][q]) : 0.0;
+        }
+#pragma unroll
+        for (int h = 0; h < H; ++h) {
+            const int t = lane + h * S;
+            const int k0 = ((b >> 2) + t) << 2;
+#pragma unroll
+            for (int q = 0; q < 4; ++q)
+                if (t < trip && k0 + q >= b && k0 + q < e) acc = fma(v[h][q], xv[h][q], acc);
+        }
+        for (int t = lane + H * S; t < trip; t += S) {
+            const int k0 = ((b >> 2) + t) << 2;
+            int cc[4];
+            double vv[4];
+            if (k0 + 4 <= nnz) {
+                ld_quad<0>(col + k0, val + k0, 0, cc, vv);
+            } else {
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    const int kq = min(k0 + q, nnz - 1);
+                    cc[q] = __ldg(col + kq);
+                    vv[q] = __ldg(val + kq);
+                }
+            }
+#pragma unroll
+            for (int q = 0; q < 4; ++q)
+                if (k0 + q >= b && k0 + q < e) acc = fma(vv[q], __ldg(x + cc[q]), acc);
+        }
+#pragma unroll
+        for (int off = S / 2; off >= 1; off >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, off);
+        if (lane == 0) y[i] = acc;
+    }
+}
+
 __global__ void flush_kernel(int4* p, size_t n) {
     for (size_t k = blockIdx.x * (size_t)blockDim.x + threadIdx.x; k < n; k += (size_t)gridDim.x * blockDim.x)
         p[k] = make_int4((int)k, 1, 2, 3);
@@ -580,14 +651,15 @@ int main(int argc, char** argv) {
     } vs[] = {
         {"S2 quads ldg (headline)", spmv_q<2, 0>, 1024, 0, "q"},
         {"S2 quads apw 63MB", spmv_q<2, 0>, 1024, 0, nullptr, 63},
-        {"win C2048 H2048", spmv_win<2, 2048, 2048>, 1024, (2048 + 4096 + 2) * 8, nullptr, 0, 2048},
-        {"win C4096 H2048", spmv_win<2, 4096, 2048>, 1024, (4096 + 4096 + 2) * 8, nullptr, 0, 4096},
-        {"win C2048 H4096", spmv_win<2, 2048, 4096>, 1024, (2048 + 8192 + 2) * 8, nullptr, 0, 2048},
-        {"win C4096 H4096", spmv_win<2, 4096, 4096>, 1024, (4096 + 8192 + 2) * 8, nullptr, 0, 4096},
-        {"win C8192 H2048", spmv_win<2, 8192, 2048>, 1024, (8192 + 4096 + 2) * 8, nullptr, 0, 8192},
-        {"win C4096 H2048 apw", spmv_win<2, 4096, 2048>, 1024, (4096 + 4096 + 2) * 8, nullptr, 63, 4096},
-        {"win C2048 H4096 apw", spmv_win<2, 2048, 4096>, 1024, (2048 + 8192 + 2) * 8, nullptr, 63, 2048},
-        {"win C4096 H4096 apw", spmv_win<2, 4096, 4096>, 1024, (4096 + 8192 + 2) * 8, nullptr, 63, 4096},
+        {"qh S2 H1 1024x2", spmv_qh<2, 1, 1024, 2>},
+        {"qh S2 H2 1024x2", spmv_qh<2, 2, 1024, 2>},
+        {"qh S2 H2 768x2", spmv_qh<2, 2, 768, 2>, 768},
+        {"qh S2 H2 512x3", spmv_qh<2, 2, 512, 3>, 512},
+        {"qh S2 H2 1024x1", spmv_qh<2, 2, 1024, 1>},
+        {"qh S2 H2 768x2 apw", spmv_qh<2, 2, 768, 2>, 768, 0, nullptr, 63},
+        {"qh S2 H2 512x3 apw", spmv_qh<2, 2, 512, 3>, 512, 0, nullptr, 63},
+        {"qh S2 H1 1024x2 apw", spmv_qh<2, 1, 1024, 2>, 1024, 0, nullptr, 63},
+        {"qh S1 H2 768x2 apw", spmv_qh<1, 2, 768, 2>, 768, 0, nullptr, 63},
     };
     int k = 0;
     for (auto& v : vs) {
