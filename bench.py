@@ -404,7 +404,10 @@ def run_gpu_single(args, local_rank):
             continue
         sweep.append((ms_c, c))
     sweep.sort(key=lambda q: q[0])
-    best = min((q for q in sweep if q[1][0] >= 2), key=lambda q: q[0])[1] if args.autotune else HEADLINE
+    ran = {c for _, c in sweep}
+    # the fixed headline, unless this device cannot run it (then the best 3-level candidate)
+    best = HEADLINE if HEADLINE in ran and not args.autotune else \
+        min((q for q in sweep if q[1][0] >= 2), key=lambda q: q[0])[1]
     s1 = min((q for q in sweep if q[1][0] == 1), key=lambda q: q[0])[1]
     cfg = cfg_of(best)
     step = lambda: P.spmv_csr_f64(*t, d_y, **cfg)

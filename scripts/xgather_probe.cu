@@ -116,6 +116,11 @@ __device__ __forceinline__ void ld_quad(const int* col, const double* val, uint6
         const int4 cc = __ldg(reinterpret_cast<const int4*>(col));
         c[0] = cc.x, c[1] = cc.y, c[2] = cc.z, c[3] = cc.w;
         asm("ld.global.nc.v4.f64 {%0, %1, %2, %3}, [%4];" : "=d"(v[0]), "=d"(v[1]), "=d"(v[2]), "=d"(v[3]) : "l"(val));
+    } else if constexpr (PC == 9) {   // L1::evict_first only (CSR lines leave L1 before the x band)
+        asm("ld.global.nc.L1::evict_first.v4.s32 {%0, %1, %2, %3}, [%4];"
+            : "=r"(c[0]), "=r"(c[1]), "=r"(c[2]), "=r"(c[3]) : "l"(col));
+        asm("ld.global.nc.L1::evict_first.v4.f64 {%0, %1, %2, %3}, [%4];"
+            : "=d"(v[0]), "=d"(v[1]), "=d"(v[2]), "=d"(v[3]) : "l"(val));
     } else if constexpr (PC == 7) {   // L1::no_allocate only (L1 kept for the x band)
         asm("ld.global.nc.L1::no_allocate.v4.s32 {%0, %1, %2, %3}, [%4];"
             : "=r"(c[0]), "=r"(c[1]), "=r"(c[2]), "=r"(c[3]) : "l"(col));
@@ -651,15 +656,10 @@ int main(int argc, char** argv) {
     } vs[] = {
         {"S2 quads ldg (headline)", spmv_q<2, 0>, 1024, 0, "q"},
         {"S2 quads apw 63MB", spmv_q<2, 0>, 1024, 0, nullptr, 63},
-        {"qh S2 H1 1024x2", spmv_qh<2, 1, 1024, 2>},
-        {"qh S2 H2 1024x2", spmv_qh<2, 2, 1024, 2>},
-        {"qh S2 H2 768x2", spmv_qh<2, 2, 768, 2>, 768},
-        {"qh S2 H2 512x3", spmv_qh<2, 2, 512, 3>, 512},
-        {"qh S2 H2 1024x1", spmv_qh<2, 2, 1024, 1>},
-        {"qh S2 H2 768x2 apw", spmv_qh<2, 2, 768, 2>, 768, 0, nullptr, 63},
-        {"qh S2 H2 512x3 apw", spmv_qh<2, 2, 512, 3>, 512, 0, nullptr, 63},
-        {"qh S2 H1 1024x2 apw", spmv_qh<2, 1, 1024, 2>, 1024, 0, nullptr, 63},
-        {"qh S1 H2 768x2 apw", spmv_qh<1, 2, 768, 2>, 768, 0, nullptr, 63},
+        {"apw csr L1ef", spmv_q<2, 0, 9>, 1024, 0, nullptr, 63},
+        {"apw x L1el", spmv_q<2, 5, 0>, 1024, 0, nullptr, 63},
+        {"apw csr L1ef x L1el", spmv_q<2, 5, 9>, 1024, 0, nullptr, 63},
+        {"csr L1ef", spmv_q<2, 0, 9>},
     };
     int k = 0;
     for (auto& v : vs) {
