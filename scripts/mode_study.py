@@ -27,6 +27,22 @@ for S in (1, 2, 8, 32):
         runs.append(("spmv_cfg2_blocked_scalar", S, mode,
                      lambda S=S, mode=mode: P.spmv_csr_f64(*t, y, simdlen=S, mode=mode, threads_per_team=1024,
                                                            blocked=True)))
+# the 128-bit quad body (the bench headline's, without the persisting window: ncu neutralises it)
+for S in (1, 2, 4, 8):
+    for mode in (("spmd",) if S == 1 else ("spmd", "generic_smem", "generic_shfl")):
+        runs.append(("spmv_cfg2_blocked_quads", S, mode,
+                     lambda S=S, mode=mode: P.spmv_csr_f64(*t, y, simdlen=S, mode=mode, threads_per_team=1024,
+                                                           blocked=True, quad=True)))
+# transpose-reduce: SPMD with two rows per group in flight
+for S in (8, 16):
+    runs.append(("spmv_cfg2_blocked_pairs_U2", S, "spmd",
+                 lambda S=S: P.spmv_csr_f64(*t, y, simdlen=S, mode="spmd", threads_per_team=1024, blocked=True,
+                                            vec128=True, outer_unroll=2)))
+for S in (1, 4, 8, 32):
+    for mode in (("spmd",) if S == 1 else ("spmd", "generic_smem", "generic_shfl")):
+        runs.append((f"stencil_pairs_N2^20_L{L}", S, mode,
+                     lambda S=S, mode=mode: P.nested_stencil_f64(inp, coef, w, N, L, out, visits, simdlen=S,
+                                                                 mode=mode, vec128=True, blocked=True)))
 for S in (1, 4, 8, 32):
     for mode in (("spmd",) if S == 1 else ("spmd", "generic_smem", "generic_shfl")):
         runs.append((f"stencil_N2^20_L{L}", S, mode,
