@@ -36,7 +36,12 @@ build/%.o: $(CSRC)/%.cu $(CU_HDRS)
 $(PKG)/libnest.so: $(CU_OBJS)
 	$(NVCC) $(ARCH) $(NVLINK) -o $@ $(CU_OBJS)
 
+# the C ABI from plain C (examples/spmv_c.c): gcc + libnest.so + the CUDA runtime
+examples/spmv_c: examples/spmv_c.c include/nest.h $(PKG)/libnest.so
+	$(CC) -O2 -Wall -Iinclude -I/usr/local/cuda/include -o $@ $< -L$(PKG) -lnest \
+	    -Wl,-rpath,'$$ORIGIN/../$(PKG)' -L/usr/local/cuda/lib64 -lcudart -Wl,-rpath,/usr/local/cuda/lib64
+
 clean:
-	rm -rf build nestgen/libnestgen.so oracle/liboracle.so $(PKG)/libnest.so
+	rm -rf build nestgen/libnestgen.so oracle/liboracle.so $(PKG)/libnest.so examples/spmv_c
 
 .PHONY: all host clean

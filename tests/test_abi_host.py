@@ -251,3 +251,15 @@ def test_x_l2_persist_flag_rules():
     assert N.NEST_F_X_L2_PERSIST == 1 << 6
     with open(os.path.join(ROOT, "include", "nest.h")) as f:
         assert "NEST_F_X_L2_PERSIST = 1u << 6" in f.read()
+
+
+def test_c_example_builds_against_the_header_and_library():
+    # the boundary is a C ABI: a plain C program (examples/spmv_c.c) compiles against
+    # include/nest.h and links libnest.so with gcc alone (tests/test_gpu_parity.py runs it)
+    import subprocess
+    r = subprocess.run(["make", "-C", ROOT, "examples/spmv_c"], capture_output=True, text=True)
+    assert r.returncode == 0, r.stdout + r.stderr
+    exe = os.path.join(ROOT, "examples", "spmv_c")
+    assert os.access(exe, os.X_OK)
+    ldd = subprocess.run(["ldd", exe], capture_output=True, text=True).stdout
+    assert "libnest.so" in ldd and "not found" not in ldd, ldd

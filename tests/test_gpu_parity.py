@@ -705,3 +705,15 @@ def test_spmv_x_l2_persist_plan_and_flush(P, banded):
     assert during > 0 and info["l2_setaside_bytes"] > 0
     P.shutdown()
     assert lim() < during
+
+
+def test_c_example_runs(P):
+    # examples/spmv_c.c: the headline and a generic-SMEM configuration through the C ABI from
+    # plain C, bit-exact against a C loop on integer-valued data (exit status 0)
+    import os
+    import subprocess
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    assert subprocess.run(["make", "-C", root, "examples/spmv_c"], capture_output=True).returncode == 0
+    r = subprocess.run([os.path.join(root, "examples", "spmv_c")], capture_output=True, text=True, timeout=300)
+    assert r.returncode == 0, r.stdout + r.stderr
+    assert r.stdout.count(": 0 mismatching rows") == 2, r.stdout
