@@ -19,6 +19,7 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--Ls", default="4,8,16,32,64")
 ap.add_argument("--iters", type=int, default=15)
 ap.add_argument("--json", default="")
+ap.add_argument("--U", default="1", help="outer_unroll values (SPMD transpose-reduce), e.g. 1,2,4")
 a = ap.parse_args()
 N = 1 << 20
 flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
@@ -30,10 +31,11 @@ for L in map(int, a.Ls.split(",")):
     B = 8 * (N * L + 2) + 16 * N + 8 * L
     for S in (1, 2, 4, 8, 16):
         for unit in ("scalar", "pairs"):
-            for T in (256, 512, 1024):
-                for blocked in (False, True):
+            for T, blocked, U in ((T, b, U) for T in (256, 512, 1024) for b in (False, True)
+                                  for U in map(int, a.U.split(","))):
+                if True:
                     cfg = dict(simdlen=S, mode="spmd", threads_per_team=T, blocked=blocked,
-                               vec128=unit != "scalar")
+                               vec128=unit != "scalar", outer_unroll=U)
                     try:
                         P.nested_stencil_f64(*t, N, L, o, **cfg)
                     except P.NestError:
@@ -53,7 +55,7 @@ for L in map(int, a.Ls.split(",")):
     best = min(rows, key=lambda r: r["ms"])
     s1 = min((r for r in rows if r["simdlen"] == 1), key=lambda r: r["ms"])
     print(f"L={L:3d} best {best['GBs']:7.1f} GB/s ({best['GBs'] / 6446:.3f}) S={best['simdlen']} {best['unit']} "
-          f"T={best['threads_per_team']} blocked={best['blocked']}  | simdlen1 {s1['GBs']:7.1f} ({s1['unit']} "
+          f"T={best['threads_per_team']} blocked={best['blocked']} U={best['outer_unroll']}  | simdlen1 {s1['GBs']:7.1f} ({s1['unit']} "
           f"T={s1['threads_per_team']})  speedup {s1['ms'] / best['ms']:.2f}", flush=True)
     for unit in ("scalar", "pairs"):
         ur = [r for r in rows if r["unit"] == unit]
