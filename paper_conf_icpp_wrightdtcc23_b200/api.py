@@ -35,6 +35,13 @@ def make_desc(simdlen: int = 8, mode: str | int = "spmd", reduce: str | int = "s
               x_halo: int = 0, blocked: bool = False,
               vec128: bool = False, quad: bool = False, team_chunk: int = 0, teams_per_sm: int = 0,
               x_l2_persist: bool = False, flags: int = 0) -> N.nest_desc:
+    """A nest_desc (include/nest.h) from keyword arguments: the integer fields by name
+    (simdlen, threads_per_team, num_teams, sharing_bytes, outer_unroll, x_halo,
+    team_chunk, teams_per_sm), mode "spmd" / "generic_smem" / "generic_shfl" /
+    "teams_generic", reduce "sum" / "max" / "min", and the flags: persistent ->
+    NEST_F_PERSISTENT_GRID, stream_hints -> NEST_F_STREAM_HINTS, blocked -> NEST_F_BLOCKED,
+    vec128 -> NEST_F_VEC128, quad -> NEST_F_VEC128 | NEST_F_VEC_QUAD, x_l2_persist ->
+    NEST_F_X_L2_PERSIST (plus any raw bits in `flags`)."""
     d = N.nest_desc()
     d.abi_version = N.NEST_ABI_VERSION
     d.num_teams = num_teams
