@@ -55,6 +55,9 @@ CONFIGS = {
     "pshape": [(f"S{S} {'quads' if q else 'pairs'} T{T} persist", dict(simdlen=S, vec128=True, quad=q, blocked=True,
                                                                       threads_per_team=T, x_l2_persist=True))
                for S in (2, 4) for q in (True, False) for T in (512, 640, 768, 1024)],
+    "waves": [(f"S2 quads persist teams {nt}", dict(simdlen=2, quad=True, blocked=True, threads_per_team=1024,
+                                                    x_l2_persist=True, num_teams=nt))
+              for nt in (0, 592, 888, 1184, 2368, 4736)],
     "cfg5ab": [(f"S8 {nm} rep{r}", dict(simdlen=8, vec128=True, quad=q, blocked=True, threads_per_team=1024))
                for r in range(3) for nm, q in (("pairs", False), ("quads", True))],
     "cfg5": [(f"S{S} {'quads' if q else 'pairs'} U{U}{' persist' if pe else ''}",

@@ -593,6 +593,113 @@ __global__ void __launch_bounds__(TB, MINB)
     }
 }
 
+// Per-team start / end times (%globaltimer, ns) of the headline structure: how much of the
+// kernel is the tail after the median team has finished?
+__device__ unsigned long long g_t0[1024], g_t1[1024];
+template <int S>
+__global__ void __launch_bounds__(1024, 2)
+    spmv_qt(const int64_t* __restrict__ rp, const int* __restrict__ col, const double* __restrict__ val,
+            const double* __restrict__ x, double* __restrict__ y, int n, int chunk, int nnz) {
+    unsigned long long t;
+    if (threadIdx.x == 0) {
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        g_t0[blockIdx.x] = t;
+    }
+    const int G = blockDim.x / S;
+    const int g = threadIdx.x / S, lane = threadIdx.x % S;
+    const int cs = blockIdx.x * chunk;
+    const int ce = min(n, cs + chunk);
+    for (int i = cs + g; i < ce; i += G) {
+        const int b = (int)__ldg(rp + i), e = (int)__ldg(rp + i + 1);
+        const int trip = e > b ? ((e + 3) >> 2) - (b >> 2) : 0;
+        double acc = 0.0;
+        for (int tt = lane; tt < trip; tt += S) {
+            const int k0 = ((b >> 2) + tt) << 2;
+            int c[4];
+            double v[4];
+            if (k0 + 4 <= nnz) {
+                ld_quad<0>(col + k0, val + k0, 0, c, v);
+            } else {
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    const int kq = k0 + q < nnz ? k0 + q : k0;
+                    c[q] = __ldg(col + kq);
+                    v[q] = __ldg(val + kq);
+                }
+            }
+#pragma unroll
+            for (int q = 0; q < 4; ++q)
+                if (k0 + q >= b && k0 + q < e) acc = fma(v[q], __ldg(x + c[q]), acc);
+        }
+#pragma unroll
+        for (int off = S / 2; off >= 1; off >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, off);
+        if (lane == 0) y[i] = acc;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        g_t1[blockIdx.x] = t;
+    }
+}
+
+// Tail pool (experiment): team b's first (1 - F/100) of its chunk is processed as in the
+// headline (static); the last F% of every chunk forms one global pool of 16-row warp
+// blocks (round-robin over the teams), claimed by any warp that has finished its own part
+// (one atomicAdd per block on g_pool, zeroed before every launch).  Results identical (a
+// row is computed the same way by whichever warp takes it).
+__device__ int g_pool;
+template <int S, int F>
+__global__ void __launch_bounds__(1024, 2)
+    spmv_qpool(const int64_t* __restrict__ rp, const int* __restrict__ col, const double* __restrict__ val,
+               const double* __restrict__ x, double* __restrict__ y, int n, int chunk, int nnz) {
+    constexpr int RB = 32 / S;   // rows per warp block
+    const int W = blockDim.x / 32, w = threadIdx.x / 32;
+    const int gl = (threadIdx.x & 31) / S, lane = threadIdx.x % S;
+    const int nblk_team = chunk / RB;                       // chunk is a multiple of G (so of RB)
+    const int tail = (nblk_team * F / 100 + W - 1) / W * W; // pool blocks per team
+    const int priv = nblk_team - tail;
+    auto row_block = [&](int team, int j) {
+        const int r0 = team * chunk + j * RB;
+        const int i = r0 + gl;
+        if (i >= n) return;
+        const int b = (int)__ldg(rp + i), e = (int)__ldg(rp + i + 1);
+        const int trip = e > b ? ((e + 3) >> 2) - (b >> 2) : 0;
+        double acc = 0.0;
+        for (int t = lane; t < trip; t += S) {
+            const int k0 = ((b >> 2) + t) << 2;
+            int c[4];
+            double v[4];
+            if (k0 + 4 <= nnz) {
+                ld_quad<0>(col + k0, val + k0, 0, c, v);
+            } else {
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    const int kq = k0 + q < nnz ? k0 + q : k0;
+                    c[q] = __ldg(col + kq);
+                    v[q] = __ldg(val + kq);
+                }
+            }
+#pragma unroll
+            for (int q = 0; q < 4; ++q)
+                if (k0 + q >= b && k0 + q < e) acc = fma(v[q], __ldg(x + c[q]), acc);
+        }
+#pragma unroll
+        for (int off = S / 2; off >= 1; off >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, off);
+        if (lane == 0) y[i] = acc;
+    };
+    for (int j = w; j < priv; j += W) row_block(blockIdx.x, j);
+    const int total = tail * gridDim.x;
+    while (true) {
+        int q = 0;
+        if ((threadIdx.x & 31) == 0) q = atomicAdd(&g_pool, 1);
+        q = __shfl_sync(0xffffffffu, q, 0);
+        if (q >= total) break;
+        row_block(q % gridDim.x, priv + q / gridDim.x);
+    }
+}
+
+__global__ void zero_pool() { g_pool = 0; }
+
 __global__ void flush_kernel(int4* p, size_t n) {
     for (size_t k = blockIdx.x * (size_t)blockDim.x + threadIdx.x; k < n; k += (size_t)gridDim.x * blockDim.x)
         p[k] = make_int4((int)k, 1, 2, 3);
@@ -656,10 +763,11 @@ int main(int argc, char** argv) {
     } vs[] = {
         {"S2 quads ldg (headline)", spmv_q<2, 0>, 1024, 0, "q"},
         {"S2 quads apw 63MB", spmv_q<2, 0>, 1024, 0, nullptr, 63},
-        {"apw csr L1ef", spmv_q<2, 0, 9>, 1024, 0, nullptr, 63},
-        {"apw x L1el", spmv_q<2, 5, 0>, 1024, 0, nullptr, 63},
-        {"apw csr L1ef x L1el", spmv_q<2, 5, 9>, 1024, 0, nullptr, 63},
-        {"csr L1ef", spmv_q<2, 0, 9>},
+        {"pool 3% apw", spmv_qpool<2, 3>, 1024, 0, nullptr, 63},
+        {"pool 6% apw", spmv_qpool<2, 6>, 1024, 0, nullptr, 63},
+        {"pool 10% apw", spmv_qpool<2, 10>, 1024, 0, nullptr, 63},
+        {"pool 20% apw", spmv_qpool<2, 20>, 1024, 0, nullptr, 63},
+        {"S2 quads apw 63MB (again)", spmv_q<2, 0>, 1024, 0, nullptr, 63},
     };
     int k = 0;
     for (auto& v : vs) {
@@ -690,6 +798,7 @@ int main(int argc, char** argv) {
         for (int r = 0; r < 13; ++r) {
             if (v.apw) CK(cudaCtxResetPersistingL2Cache());
             flush_kernel<<<4 * prop.multiProcessorCount, 1024, 0, st>>>(fl, flush_bytes / 16);
+            if (strstr(v.name, "pool")) zero_pool<<<1, 1, 0, st>>>();
             CK(cudaEventRecord(e0, st));
             v.fn<<<grid, v.T, v.smem, st>>>(drp, dcol, dval, dx, dy, n, chunk, nnz);
             CK(cudaEventRecord(e1, st));
@@ -721,6 +830,23 @@ int main(int argc, char** argv) {
         }
         printf("%2d %-28s grid %4d median %.4f ms min %.4f  %.0f GB/s alg  %s\n", k, v.name, grid, med, ts[0],
                alg / med * 1e-6, tag);
+        if (strstr(v.name, "timed")) {
+            std::vector<unsigned long long> t0(grid), t1(grid);
+            CK(cudaMemcpyFromSymbol(t0.data(), g_t0, grid * 8));
+            CK(cudaMemcpyFromSymbol(t1.data(), g_t1, grid * 8));
+            const unsigned long long base = *std::min_element(t0.begin(), t0.end());
+            std::vector<double> st(grid), en(grid);
+            for (int q = 0; q < grid; ++q) st[q] = (t0[q] - base) * 1e-3, en[q] = (t1[q] - base) * 1e-3;
+            std::sort(st.begin(), st.end());
+            std::sort(en.begin(), en.end());
+            if (getenv("XG_DUMP")) {
+                FILE* f = fopen(getenv("XG_DUMP"), "w");
+                for (int q = 0; q < grid; ++q) fprintf(f, "%d %.2f %.2f\n", q, (t0[q] - base) * 1e-3, (t1[q] - base) * 1e-3);
+                fclose(f);
+            }
+            printf("   team start us: min %.1f median %.1f max %.1f | team end us: min %.1f p10 %.1f median %.1f p90 %.1f max %.1f\n",
+                   st[0], st[grid / 2], st[grid - 1], en[0], en[grid / 10], en[grid / 2], en[grid * 9 / 10], en[grid - 1]);
+        }
     }
     // ---- DRAM-side diagnostic (stream_gather); time here, bytes under ncu
     typedef void (*SgFn)(const int*, const double*, const double*, int, double*);
