@@ -1,0 +1,99 @@
+"""Property-based GPU parity (hypothesis, derandomised): random small CSR matrices with
+integer data (exact in fp64, so the bar is bit-exactness, R4) against the
+oracle, under random launch configurations -- simdlen, mode, team size, outer unroll,
+schedule (cyclic / blocked / team chunks), loads (scalar / pairs / quads), explicit
+team counts, small sharing spaces (global fallback), the x ring and the persisting
+window.  Configurations the library rejects as NEST_ERR_UNSUPPORTED (a variant's
+register-limited team size) are skipped; anything else must match bit for bit."""
+import numpy as np
+import pytest
+from hypothesis import assume, given, settings, strategies as st
+
+import oracle
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+SET = settings(max_examples=600, deadline=None, derandomize=True)
+
+
+@pytest.fixture(scope="module")
+def P():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_icpp_wrightdtcc23_b200 as P
+    return P
+
+
+@st.composite
+def int_csr(draw):
+    nrows = draw(st.integers(0, 3000))
+    ncols = draw(st.integers(1, 5000))
+    long_rows = draw(st.booleans())
+    seed = draw(st.integers(0, 2**32 - 1))
+    rng = np.random.default_rng(seed)
+    lens = rng.integers(0, 80 if long_rows else 14, nrows)
+    lens = np.minimum(lens, ncols)
+    rp = np.zeros(nrows + 1, np.int64)
+    rp[1:] = np.cumsum(lens)
+    col = np.empty(int(rp[-1]), np.int32)
+    for i in range(nrows):
+        col[rp[i]:rp[i + 1]] = np.sort(rng.choice(ncols, int(lens[i]), replace=False))
+    val = rng.integers(-7, 8, col.size).astype(np.float64)
+    x = rng.integers(-7, 8, ncols).astype(np.float64)
+    return rp, col, val, x
+
+
+@st.composite
+def launch(draw):
+    S = draw(st.sampled_from([1, 2, 4, 8, 16, 32]))
+    cfg = dict(simdlen=S, mode=draw(st.sampled_from(["spmd", "generic_smem", "generic_shfl"])),
+               threads_per_team=draw(st.sampled_from([32, 64, 128, 256, 512, 768, 1024])),
+               outer_unroll=draw(st.sampled_from([1, 1, 2, 4])),
+               sharing_bytes=draw(st.sampled_from([0, 0, 64, 256])),
+               num_teams=draw(st.sampled_from([0, 0, 1, 3, 7])))
+    loads = draw(st.sampled_from(["scalar", "pairs", "quads"]))
+    cfg["vec128"], cfg["quad"] = loads != "scalar", loads == "quads"
+    kind = draw(st.sampled_from(["cyclic", "blocked", "chunks", "ring", "persist"]))
+    if kind == "blocked":
+        cfg["blocked"] = True
+    elif kind == "chunks":
+        cfg.update(blocked=True, team_chunk=draw(st.sampled_from([1, 64, 1000])))
+    elif kind == "ring":
+        cfg["x_halo"] = draw(st.sampled_from([1, 64, 700]))
+        cfg["threads_per_team"] = max(64, cfg["threads_per_team"])
+    else:
+        cfg.update(blocked=draw(st.booleans()), x_l2_persist=kind == "persist")
+    return cfg
+
+
+def bits(a):
+    return np.ascontiguousarray(a).view(np.int64)
+
+
+@SET
+@given(int_csr(), launch())
+def test_spmv_random_matrices_and_launches_bit_exact(P, m, cfg):
+    rp, col, val, x = m
+    yref, _ = oracle.spmv_csr_f64(rp, col, val, x)
+    t = [torch.from_numpy(a).cuda() for a in (rp, col, val, x)]
+    try:
+        y = P.spmv_csr_f64(*t, **cfg).cpu().numpy()
+    except P.NestError as e:
+        assume(e.status != P._nest.NEST_ERR_UNSUPPORTED)
+        raise
+    assert np.array_equal(bits(y), bits(yref)), cfg
+
+
+@SET
+@given(int_csr(), st.sampled_from(["max", "min"]), launch())
+def test_spmv_random_max_min(P, m, op, cfg):
+    rp, col, val, x = m
+    yref, _ = oracle.spmv_csr_f64(rp, col, val, x, op=op)
+    t = [torch.from_numpy(a).cuda() for a in (rp, col, val, x)]
+    try:
+        y = P.spmv_csr_f64(*t, reduce=op, **cfg).cpu().numpy()
+    except P.NestError as e:
+        assume(e.status != P._nest.NEST_ERR_UNSUPPORTED)
+        raise
+    assert np.array_equal(y, yref), cfg   # by value: the sign of a zero tie is unordered (R17)
