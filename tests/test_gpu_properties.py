@@ -97,3 +97,64 @@ def test_spmv_random_max_min(P, m, op, cfg):
         assume(e.status != P._nest.NEST_ERR_UNSUPPORTED)
         raise
     assert np.array_equal(y, yref), cfg   # by value: the sign of a zero tie is unordered (R17)
+
+
+@st.composite
+def body_launch(draw):
+    S = draw(st.sampled_from([1, 2, 4, 8, 16, 32]))
+    return dict(simdlen=S, mode=draw(st.sampled_from(["spmd", "generic_smem", "generic_shfl"])),
+                threads_per_team=draw(st.sampled_from([32, 128, 256, 512, 1024])),
+                outer_unroll=draw(st.sampled_from([1, 1, 2, 4])),
+                sharing_bytes=draw(st.sampled_from([0, 0, 64])),
+                num_teams=draw(st.sampled_from([0, 0, 1, 5])),
+                blocked=draw(st.booleans()), vec128=draw(st.booleans()))
+
+
+def _run(P, fn):
+    try:
+        return fn()
+    except P.NestError as e:
+        assume(e.status != P._nest.NEST_ERR_UNSUPPORTED)
+        raise
+
+
+@settings(max_examples=300, deadline=None, derandomize=True)
+@given(st.integers(0, 5000), st.integers(1, 70), st.integers(0, 2**32 - 1), body_launch())
+def test_stencil_random_bit_exact_and_visits(P, N, L, seed, cfg):
+    # a10: integer data (exact), the guarded side effect counted once per outer iteration
+    from nestgen import recipes as R
+    if cfg["vec128"] and L % 2:
+        L += 1
+    inp, coef, w = R.stencil_inputs(N, L, values="int", cfg_seed=seed % 100000)
+    yref, _, vref = oracle.nested_stencil_f64(inp, coef, w, N, L)
+    visits = torch.zeros(1, dtype=torch.int64, device="cuda")
+    t = [torch.from_numpy(a).cuda() for a in (inp, coef, w)]
+    out = _run(P, lambda: P.nested_stencil_f64(*t, N, L, visits=visits, **cfg)).cpu().numpy()
+    assert np.array_equal(bits(out), bits(yref)) and int(visits.item()) == vref == N, cfg
+
+
+@settings(max_examples=200, deadline=None, derandomize=True)
+@given(st.integers(0, 400), st.sampled_from([1, 3, 16, 64]), st.sampled_from([4, 8, 36, 64]),
+       st.integers(0, 2**32 - 1), body_launch())
+def test_batched_random_bit_exact(P, B, m, n, seed, cfg):
+    # a9: integer data (partial sums < 2^24: exact in fp32), any m x n
+    from nestgen import recipes as R
+    A, x = R.batched_inputs(B, m, n, values="int", cfg_seed=seed % 100000)
+    yref, _ = oracle.batched_matvec_f32(A, x, B, m, n)
+    y = _run(P, lambda: P.batched_matvec_f32(torch.from_numpy(A).cuda(), torch.from_numpy(x).cuda(), B, m, n,
+                                             **cfg)).cpu().numpy()
+    assert np.array_equal(y.view(np.int32), yref.view(np.int32)), cfg
+
+
+@settings(max_examples=150, deadline=None, derandomize=True)
+@given(st.integers(1, 12), st.integers(1, 12), st.integers(1, 70), st.integers(0, 2**32 - 1), body_launch())
+def test_laplace_random_bit_exact(P, nz, ny, nx, seed, cfg):
+    # NEXT-2 (R21): bit-identical to the oracle, boundary points untouched
+    from nestgen import recipes as R
+    if cfg["vec128"] and nx % 2:
+        nx += 1
+    u = R.laplace_inputs(nz, ny, nx, values="real", cfg_seed=seed % 100000)
+    ref = oracle.laplace3d_f64(u, nz, ny, nx, 0.125)
+    out = torch.from_numpy(u.copy()).cuda()
+    _run(P, lambda: P.laplace3d_f64(torch.from_numpy(u).cuda(), out, nz, ny, nx, 0.125, **cfg))
+    assert np.array_equal(bits(out.cpu().numpy()), bits(ref)), cfg
