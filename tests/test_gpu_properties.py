@@ -158,3 +158,34 @@ def test_laplace_random_bit_exact(P, nz, ny, nx, seed, cfg):
     out = torch.from_numpy(u.copy()).cuda()
     _run(P, lambda: P.laplace3d_f64(torch.from_numpy(u).cuda(), out, nz, ny, nx, 0.125, **cfg))
     assert np.array_equal(bits(out.cpu().numpy()), bits(ref)), cfg
+
+
+@settings(max_examples=120, deadline=None, derandomize=True)
+@given(int_csr(), st.integers(1, 8), st.sampled_from([1, 2, 4, 8, 32]),
+       st.sampled_from(["spmd", "generic_smem", "generic_shfl"]), st.booleans(), st.booleans())
+def test_xpeer_random_virtual_ranks(P, m, nranks, S, mode, vec, blocked):
+    # NEXT-4 on virtual ranks: every rank's rows, gathering x from the owners' slices,
+    # bit-exact against the oracle (integer data)
+    rp, col, val, x = m
+    n = rp.size - 1
+    ncols = x.size
+    yref, _ = oracle.spmv_csr_f64(rp, col, val, x)
+    xc = P.x_chunk(ncols, nranks)
+    sl = []
+    for r in range(nranks):
+        s = torch.zeros(max(xc, 1), dtype=torch.float64, device="cuda")
+        b, k = P.local_x_range(ncols, nranks, r)
+        if k > 0:
+            s[:k] = torch.from_numpy(x[b:b + k]).cuda()
+        sl.append(s)
+    for r in range(nranks):
+        _, rb, nloc = P.shard_rows(n, nranks, r)
+        lrp = rp[rb:rb + nloc + 1] - rp[rb]
+        t = [torch.from_numpy(np.ascontiguousarray(a)).cuda()
+             for a in (lrp, col[rp[rb]:rp[rb + nloc]], val[rp[rb]:rp[rb + nloc]])]
+        xp = P.XPeer(ncols, nranks=nranks, rank=r, local_slices=sl)
+        try:
+            y = _run(P, lambda: xp.spmv_csr_f64(n, *t, simdlen=S, mode=mode, vec128=vec, blocked=blocked))
+        finally:
+            xp.close()
+        assert np.array_equal(bits(y.cpu().numpy()), bits(yref[rb:rb + nloc])), (nranks, r, S, mode, vec)
