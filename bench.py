@@ -464,6 +464,7 @@ def run_gpu_single(args, local_rank):
         for c in heads:
             lms = time_leg(torch, P, lspec, c, lt, ly, flush, 10)
             leg["configs"][json.dumps(list(c))] = {"ms": lms, "GBs": LB / (lms / 1e3) / 1e9,
+                                                   "gflops": 2 * lnnz / (lms / 1e3) / 1e9,
                                                    "roofline": roofline(LB, lms, peak, peak_src, c, lspec),
                                                    "parity": parity(ly.cpu().numpy(), lyref, laref)}
         h3 = leg["configs"][json.dumps(list(heads[0]))]
@@ -486,6 +487,8 @@ def run_gpu_single(args, local_rank):
                          "lines)",
                    "parallelism": "1 GPU"},
         "parity": par,
+        "gflops": 2 * nnz / (ms / 1e3) / 1e9,
+        "gflops_rule": "2 flops (multiply + add) per nonzero",
         "speedup_vs_simdlen1": ms1 / ms,
         "simdlen1": {"ms_per_step": ms1, "GBs": B / (ms1 / 1e3) / 1e9, "config": cfg_of(s1)},
         "sweep_ms": {json.dumps(list(c)): round(m, 4) for m, c in sweep},
@@ -598,6 +601,7 @@ def run_gpu_multi(args, rank, world, local_rank):
                 "config": {"workload": workload(spec, "configs[4], row-partitioned at fixed total size"),
                            "alg_bytes": B, "parallelism": f"rows/{world}", "x_exchange": head,
                            "l2": "flushed between timed steps", **cfg},
+                "gflops": 2 * int(nnz_t.item()) / (ms / 1e3) / 1e9,
                 "parts_ms": {k: v[0] for k, v in res.items()},
                 "local_spmv_GBs_per_gpu": (B_local / (res["local_spmv_alone"][0] / 1e3) / 1e9
                                            if "local_spmv_alone" in res else None),
