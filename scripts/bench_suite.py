@@ -304,7 +304,8 @@ def cfg5(out):
 def fig9(out):
     """Fig 9 analogue: CSR SpMV time per simdlen and mode on the
     short-row cfg2 matrix and its all-far variant, best variant per (S, mode)
-    among blocked teams of 1024 with scalar / 128-bit pair / quad loads."""
+    among blocked teams of 1024 with scalar / 128-bit pair / quad loads, each with
+    and without x persisting in L2 (NEST_F_X_L2_PERSIST)."""
     res = {}
     for spec in (R.CFG2, R.CFG2_UNIFORM):
         rp, col, val = R.spmv_matrix(spec)
@@ -317,12 +318,12 @@ def fig9(out):
             for mode in (("spmd",) if S == 1 else MODES):
                 best = None
                 # U > 1 in SPMD: U rows per group in flight, reduced together (transpose-reduce)
-                variants = [(f, 1, 1024) for f in ("b", "bv", "bq")]
+                variants = [(f, 1, 1024) for f in ("b", "bv", "bq", "bp", "bvp", "bqp")]
                 if mode == "spmd" and S > 1:
-                    variants += [(f, U, T) for f in ("b", "bv") for U in (2, 4) for T in (512, 1024)]
+                    variants += [(f, U, T) for f in ("b", "bv", "bvp") for U in (2, 4) for T in (512, 1024)]
                 for flags, U, T in variants:
-                    cfg = dict(simdlen=S, mode=mode, threads_per_team=T, blocked=True, vec128=flags != "b",
-                               quad=flags == "bq", outer_unroll=U)
+                    cfg = dict(simdlen=S, mode=mode, threads_per_team=T, blocked=True, vec128="v" in flags or
+                               "q" in flags, quad="q" in flags, outer_unroll=U, x_l2_persist="p" in flags)
                     try:
                         ms = timed(lambda: P.spmv_csr_f64(*t, y, **cfg), iters=5)
                     except P.NestError:
