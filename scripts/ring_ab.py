@@ -55,6 +55,10 @@ CONFIGS = {
     "pshape": [(f"S{S} {'quads' if q else 'pairs'} T{T} persist", dict(simdlen=S, vec128=True, quad=q, blocked=True,
                                                                       threads_per_team=T, x_l2_persist=True))
                for S in (2, 4) for q in (True, False) for T in (512, 640, 768, 1024)],
+    "generic": [(f"S{S} {m} {fl} T{T}", dict(simdlen=S, mode=m, blocked=True, threads_per_team=T,
+                                               vec128=fl != "scalar", quad=fl == "quads", x_l2_persist=True))
+                for S in (2, 4, 8) for m in ("generic_smem", "generic_shfl") for fl in ("scalar", "pairs", "quads")
+                for T in (768, 1024)],
     "waves": [(f"S2 quads persist teams {nt}", dict(simdlen=2, quad=True, blocked=True, threads_per_team=1024,
                                                     x_l2_persist=True, num_teams=nt))
               for nt in (0, 592, 888, 1184, 2368, 4736)],
