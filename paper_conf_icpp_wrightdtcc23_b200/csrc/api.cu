@@ -167,7 +167,7 @@ static nest_status plan_core(const nest_desc* d, int64_t outer, int32_t K, int32
 
 nest_status make_plan(const nest_desc* d, int64_t outer, int32_t K, PayloadFn payload_of, Plan* p,
                       bool spmv_window) {
-    int32_t T, sharing, U;
+    int32_t T = 0, sharing = 0, U = 1;   // set by validate_desc on success
     nest_status s = validate_desc(d, &T, &sharing, &U);
     if (s != NEST_OK) return s;
     return plan_core(d, outer, K, T, sharing, U, payload_of(U), p, spmv_window);
@@ -175,7 +175,7 @@ nest_status make_plan(const nest_desc* d, int64_t outer, int32_t K, PayloadFn pa
 
 nest_status make_plan_fixed(const nest_desc* d, int64_t outer, int32_t K, int32_t payload, Plan* p,
                             bool spmv_window) {
-    int32_t T, sharing, U;
+    int32_t T = 0, sharing = 0, U = 1;   // set by validate_desc on success
     nest_status s = validate_desc(d, &T, &sharing, &U);
     if (s != NEST_OK) return s;
     if (payload < 0) return fail(NEST_ERR_INVALID_ARG, "payload_bytes %d < 0", payload);
