@@ -9,8 +9,8 @@ namespace nest {
 
 template <class Body, int S, int MODE, int OP>
 nest_status ring_one(const Plan& p, const RingArgs& a, cudaStream_t st) {
-    Body body{a.rowptr, a.col, a.val, XRing{a.x, nullptr, 0, 0u, 0u, (uint32_t)(a.nseg * kRingSeg)}, a.y};
-    body.nnz = a.nnz;
+    Body body{a.rowptr, a.col, a.val, XRing{a.x, nullptr, 0, 0u, 0u, (uint32_t)(a.nseg * kRingSeg)}, a.y,
+              a.nnz};
     auto* k = p.ring_tps == 2 ? spmv_ring_kernel<S, MODE, OP, 2, Body> : spmv_ring_kernel<S, MODE, OP, 1, Body>;
     cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem_bytes);
     if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(max dynamic smem)");
