@@ -700,6 +700,49 @@ __global__ void __launch_bounds__(1024, 2)
 
 __global__ void zero_pool() { g_pool = 0; }
 
+// Diagnostic (wrong values): the consumer side of a fully staged design -- row bounds
+// from global rowptr (real), each nonzero's colind / val read from a static shared "stage"
+// (k & 4095), x from a static shared window (c & 8191), and one nonzero in 16 gathering
+// x from global memory at a scattered column (the far columns).  No CSR traffic from
+// DRAM: what the consumers alone would cost if a producer kept the stages full.
+template <int S, int FAR, int TB, int MINB>
+__global__ void __launch_bounds__(TB, MINB)
+    spmv_stagediag(const int64_t* __restrict__ rp, const int* __restrict__ col, const double* __restrict__ val,
+                   const double* __restrict__ x, double* __restrict__ y, int n, int chunk, int nnz) {
+    extern __shared__ __align__(16) unsigned char sm_raw[];
+    int* scol = reinterpret_cast<int*>(sm_raw);                       // 4096 ints (16 KB)
+    double* sval = reinterpret_cast<double*>(sm_raw + 16384);        // 4096 doubles (32 KB)
+    double* xwin = reinterpret_cast<double*>(sm_raw + 16384 + 32768); // 8192 doubles (64 KB)
+    for (int k = threadIdx.x; k < 4096; k += blockDim.x) {
+        scol[k] = (int)((k * 2654435761u) & 0x7fffffff);
+        sval[k] = (double)(k & 7) - 3.0;
+    }
+    for (int k = threadIdx.x; k < 8192; k += blockDim.x) xwin[k] = (double)(k & 15);
+    __syncthreads();
+    const int G = blockDim.x / S;
+    const int g = threadIdx.x / S, lane = threadIdx.x % S;
+    const int cs = blockIdx.x * chunk;
+    const int ce = min(n, cs + chunk);
+    for (int i = cs + g; i < ce; i += G) {
+        const int b = (int)__ldg(rp + i), e = (int)__ldg(rp + i + 1);
+        double acc = 0.0;
+        for (int k = b + lane; k < e; k += S) {
+            int c;
+            double v, xv;
+            asm volatile("ld.shared.s32 %0, [%1];" : "=r"(c) : "r"(sptr(scol + (k & 4095))));
+            asm volatile("ld.shared.f64 %0, [%1];" : "=d"(v) : "r"(sptr(sval + (k & 4095))));
+            if (FAR && (k & 15) == 0)
+                xv = __ldg(x + (unsigned)c % (unsigned)n);
+            else
+                asm volatile("ld.shared.f64 %0, [%1];" : "=d"(xv) : "r"(sptr(xwin + (c & 8191))));
+            acc = fma(v, xv, acc);
+        }
+#pragma unroll
+        for (int off = S / 2; off >= 1; off >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, off);
+        if (lane == 0) y[i] = acc;
+    }
+}
+
 __global__ void flush_kernel(int4* p, size_t n) {
     for (size_t k = blockIdx.x * (size_t)blockDim.x + threadIdx.x; k < n; k += (size_t)gridDim.x * blockDim.x)
         p[k] = make_int4((int)k, 1, 2, 3);
@@ -763,11 +806,10 @@ int main(int argc, char** argv) {
     } vs[] = {
         {"S2 quads ldg (headline)", spmv_q<2, 0>, 1024, 0, "q"},
         {"S2 quads apw 63MB", spmv_q<2, 0>, 1024, 0, nullptr, 63},
-        {"pool 3% apw", spmv_qpool<2, 3>, 1024, 0, nullptr, 63},
-        {"pool 6% apw", spmv_qpool<2, 6>, 1024, 0, nullptr, 63},
-        {"pool 10% apw", spmv_qpool<2, 10>, 1024, 0, nullptr, 63},
-        {"pool 20% apw", spmv_qpool<2, 20>, 1024, 0, nullptr, 63},
-        {"S2 quads apw 63MB (again)", spmv_q<2, 0>, 1024, 0, nullptr, 63},
+        {"stagediag S2 no far 1024x1", spmv_stagediag<2, 0, 1024, 1>, 1024, 114688},
+        {"stagediag S2 far 1024x1", spmv_stagediag<2, 1, 1024, 1>, 1024, 114688, nullptr, 63},
+        {"stagediag S4 far 1024x1", spmv_stagediag<4, 1, 1024, 1>, 1024, 114688, nullptr, 63},
+        {"stagediag S1 far 1024x1", spmv_stagediag<1, 1, 1024, 1>, 1024, 114688, nullptr, 63},
     };
     int k = 0;
     for (auto& v : vs) {
