@@ -705,7 +705,7 @@ __global__ void zero_pool() { g_pool = 0; }
 // (k & 4095), x from a static shared window (c & 8191), and one nonzero in 16 gathering
 // x from global memory at a scattered column (the far columns).  No CSR traffic from
 // DRAM: what the consumers alone would cost if a producer kept the stages full.
-template <int S, int FAR, int TB, int MINB>
+template <int S, int FAR, int TB, int MINB, bool BAR = false>
 __global__ void __launch_bounds__(TB, MINB)
     spmv_stagediag(const int64_t* __restrict__ rp, const int* __restrict__ col, const double* __restrict__ val,
                    const double* __restrict__ x, double* __restrict__ y, int n, int chunk, int nnz) {
@@ -723,7 +723,11 @@ __global__ void __launch_bounds__(TB, MINB)
     const int g = threadIdx.x / S, lane = threadIdx.x % S;
     const int cs = blockIdx.x * chunk;
     const int ce = min(n, cs + chunk);
-    for (int i = cs + g; i < ce; i += G) {
+    const int rounds = (ce - cs + G - 1) / G;
+    for (int rd = 0; rd < rounds; ++rd) {
+        const int i = cs + rd * G + g;
+        if (BAR) __syncthreads();   // team-synchronous rounds (a stage per round)
+        if (i >= ce) continue;
         const int b = (int)__ldg(rp + i), e = (int)__ldg(rp + i + 1);
         double acc = 0.0;
         for (int k = b + lane; k < e; k += S) {
@@ -806,10 +810,11 @@ int main(int argc, char** argv) {
     } vs[] = {
         {"S2 quads ldg (headline)", spmv_q<2, 0>, 1024, 0, "q"},
         {"S2 quads apw 63MB", spmv_q<2, 0>, 1024, 0, nullptr, 63},
-        {"stagediag S2 no far 1024x1", spmv_stagediag<2, 0, 1024, 1>, 1024, 114688},
-        {"stagediag S2 far 1024x1", spmv_stagediag<2, 1, 1024, 1>, 1024, 114688, nullptr, 63},
-        {"stagediag S4 far 1024x1", spmv_stagediag<4, 1, 1024, 1>, 1024, 114688, nullptr, 63},
-        {"stagediag S1 far 1024x1", spmv_stagediag<1, 1, 1024, 1>, 1024, 114688, nullptr, 63},
+        {"stagediag S2 far 2x1024", spmv_stagediag<2, 1, 1024, 1>, 1024, 114688, nullptr, 63},
+        {"stagediag S2 far 1x1024 (216KB)", spmv_stagediag<2, 1, 1024, 1>, 1024, 221184, nullptr, 63},
+        {"stagediag S2 far 1x1024 rounds", spmv_stagediag<2, 1, 1024, 1, true>, 1024, 221184, nullptr, 63},
+        {"stagediag S2 far 2x1024 rounds", spmv_stagediag<2, 1, 1024, 1, true>, 1024, 114688, nullptr, 63},
+        {"stagediag S2 nofar 1x1024 rounds", spmv_stagediag<2, 0, 1024, 1, true>, 1024, 221184, nullptr, 63},
     };
     int k = 0;
     for (auto& v : vs) {
