@@ -115,7 +115,7 @@ enum {
      * 32-byte aligned val. */
     NEST_F_VEC_QUAD = 1u << 5,
     /* SpMV (nest_kernel variants: cyclic / blocked, scalar / pair / quad loads;
-     * also the dist and hostio entry points): x is marked L2-persisting for
+     * the x ring; also the dist and hostio entry points): x is marked L2-persisting for
      * this launch.  Why: the far columns of a short-row matrix gather x at
      * random, and with x (80-100 MB) competing against the streamed CSR arrays
      * for the 126 MB L2 most of those gathers miss and cost a DRAM access each
@@ -128,7 +128,7 @@ enum {
      * the caller's stream attributes are untouched.  Results are identical (a
      * cache policy only).  The persisting lines outlive the call (a following
      * SpMV on the same x finds them); nest_util_l2_flush returns them to
-     * normal, and nest_shutdown also restores the limit.  With x_halo,
+     * normal, and nest_shutdown also restores the limit.  With
      * NEST_MODE_TEAMS_GENERIC or the peer-gather SpMV: NEST_ERR_UNSUPPORTED;
      * other entry points: NEST_ERR_INVALID_ARG. */
     NEST_F_X_L2_PERSIST = 1u << 6

@@ -368,11 +368,12 @@ static nest_status spmv_plan(const nest_desc* desc, int64_t nrows, int64_t ncols
         return NEST_OK;
     }
     if (p->x_halo > 0) {
-        if (p->flags & NEST_F_X_L2_PERSIST)
-            return fail(NEST_ERR_UNSUPPORTED, "NEST_F_X_L2_PERSIST: not with the x ring (x_halo > 0)");
         *kernel = NEST_KERNEL_XRING;
         *index_bits = nnz < ((int64_t)1 << 31) - 8 && nrows < ((int64_t)1 << 31) - 8 ? 32 : 64;
-        return plan_spmv_ring(p, nrows, nnz, desc->num_teams, desc->teams_per_sm);
+        if ((s = plan_spmv_ring(p, nrows, nnz, desc->num_teams, desc->teams_per_sm)) != NEST_OK) return s;
+        if ((p->flags & NEST_F_X_L2_PERSIST) && (s = x_persist_window(p, nullptr, ncols, false)) != NEST_OK)
+            return s;
+        return NEST_OK;
     }
     *kernel = NEST_KERNEL_NEST;
     const int32_t payload = spmv_body_payload(*p, nnz);
@@ -399,14 +400,13 @@ static nest_status spmv_launch(const Plan& p, int32_t kernel, int64_t nrows, int
                                const int64_t* rowptr, const int32_t* colind, const double* val, const double* x,
                                double* y, unsigned char* fb, cudaStream_t st) {
     if (kernel == NEST_KERNEL_TEAMS_GENERIC) return launch_spmv_teams_generic(p, nrows, rowptr, colind, val, x, y, st);
-    if (kernel == NEST_KERNEL_XRING) return launch_spmv_ring(p, nrows, ncols, nnz, rowptr, colind, val, x, y, fb, st);
-    if ((p.flags & NEST_F_X_L2_PERSIST) && ncols > 0) {
-        Plan q = p;
+    Plan q = p;
+    if ((q.flags & NEST_F_X_L2_PERSIST) && ncols > 0) {   // the x window of this launch
         nest_status s = x_persist_window(&q, x, ncols, true);
         if (s != NEST_OK) return s;
-        return launch_spmv(q, (q.flags & NEST_F_STREAM_HINTS) != 0, nrows, rowptr, colind, val, x, y, fb, st, nnz);
     }
-    return launch_spmv(p, (p.flags & NEST_F_STREAM_HINTS) != 0, nrows, rowptr, colind, val, x, y, fb, st, nnz);
+    if (kernel == NEST_KERNEL_XRING) return launch_spmv_ring(q, nrows, ncols, nnz, rowptr, colind, val, x, y, fb, st);
+    return launch_spmv(q, (q.flags & NEST_F_STREAM_HINTS) != 0, nrows, rowptr, colind, val, x, y, fb, st, nnz);
 }
 
 // Alignment the variants need (checked before any launch).

@@ -38,30 +38,8 @@ nest_status launch_one(const Plan& p, const Body& body, unsigned char* fb, cudaS
         if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(max dynamic smem)");
     }
     const int64_t chunk = (p.flags & NEST_F_BLOCKED) ? p.chunk : 0;
-    if (p.l2_win) {
-        // NEST_F_X_L2_PERSIST: x under a per-launch access-policy window (the
-        // caller's stream attributes stay untouched)
-        cudaLaunchAttribute attr[1];
-        attr[0].id = cudaLaunchAttributeAccessPolicyWindow;
-        attr[0].val.accessPolicyWindow.base_ptr = const_cast<void*>(p.l2_win);
-        attr[0].val.accessPolicyWindow.num_bytes = (size_t)p.l2_win_bytes;
-        attr[0].val.accessPolicyWindow.hitRatio =
-            p.l2_setaside >= p.l2_win_bytes ? 1.0f : (float)((double)p.l2_setaside / (double)p.l2_win_bytes);
-        attr[0].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
-        attr[0].val.accessPolicyWindow.missProp = cudaAccessPropertyNormal;
-        cudaLaunchConfig_t cfg = {};
-        cfg.gridDim = dim3((unsigned)p.grid);
-        cfg.blockDim = dim3((unsigned)p.block);
-        cfg.dynamicSmemBytes = (size_t)p.smem_bytes;
-        cfg.stream = st;
-        cfg.attrs = attr;
-        cfg.numAttrs = 1;
-        const cudaError_t le = cudaLaunchKernelEx(&cfg, kern, body, p.outer, p.slot_bytes, fb, chunk);
-        if (le != cudaSuccess) return cuda_fail(le, "kernel launch (access-policy window)");
-    } else {
-        kern<<<p.grid, p.block, p.smem_bytes, st>>>(body, p.outer, p.slot_bytes, fb, chunk);
-    }
-    const cudaError_t e = cudaGetLastError();
+    const cudaError_t e = launch_with_plan(p, kern, dim3((unsigned)p.grid), dim3((unsigned)p.block),
+                                           (size_t)p.smem_bytes, st, body, p.outer, p.slot_bytes, fb, chunk);
     if (e != cudaSuccess) return cuda_fail(e, "kernel launch");
     return NEST_OK;
 }

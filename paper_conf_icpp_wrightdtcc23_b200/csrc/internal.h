@@ -59,6 +59,35 @@ inline bool spmv_index32(const Plan& p, int64_t nnz) {
 // to the set-aside (once per device) and point the window at x.
 nest_status x_persist_window(Plan* p, const double* x, int64_t ncols, bool apply);
 
+// Launch `kern` with the plan's geometry arguments; when the plan carries an x window
+// (NEST_F_X_L2_PERSIST) the launch goes through cudaLaunchKernelEx with a per-launch
+// access-policy window (hits persisting, misses normal), so the caller's stream
+// attributes stay untouched.  Returns the launch error.
+template <class Kern, class... Args>
+cudaError_t launch_with_plan(const Plan& p, Kern kern, dim3 grid, dim3 block, size_t smem, cudaStream_t st,
+                             Args... args) {
+    if (!p.l2_win) {
+        kern<<<grid, block, smem, st>>>(args...);
+        return cudaGetLastError();
+    }
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeAccessPolicyWindow;
+    attr[0].val.accessPolicyWindow.base_ptr = const_cast<void*>(p.l2_win);
+    attr[0].val.accessPolicyWindow.num_bytes = (size_t)p.l2_win_bytes;
+    attr[0].val.accessPolicyWindow.hitRatio =
+        p.l2_setaside >= p.l2_win_bytes ? 1.0f : (float)((double)p.l2_setaside / (double)p.l2_win_bytes);
+    attr[0].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+    attr[0].val.accessPolicyWindow.missProp = cudaAccessPropertyNormal;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, kern, args...);
+}
+
 // Record a thread-local error message and return `s`.
 nest_status fail(nest_status s, const char* fmt, ...) __attribute__((format(printf, 2, 3)));
 nest_status cuda_fail(cudaError_t e, const char* what);

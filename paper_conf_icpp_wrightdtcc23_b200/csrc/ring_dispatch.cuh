@@ -14,8 +14,7 @@ nest_status ring_one(const Plan& p, const RingArgs& a, cudaStream_t st) {
     auto* k = p.ring_tps == 2 ? spmv_ring_kernel<S, MODE, OP, 2, Body> : spmv_ring_kernel<S, MODE, OP, 1, Body>;
     cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, p.smem_bytes);
     if (e != cudaSuccess) return cuda_fail(e, "cudaFuncSetAttribute(max dynamic smem)");
-    k<<<p.grid, p.block, p.smem_bytes, st>>>(body, a);
-    e = cudaGetLastError();
+    e = launch_with_plan(p, k, dim3((unsigned)p.grid), dim3((unsigned)p.block), (size_t)p.smem_bytes, st, body, a);
     if (e != cudaSuccess) return cuda_fail(e, "spmv_ring launch");
     return NEST_OK;
 }

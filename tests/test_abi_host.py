@@ -242,9 +242,6 @@ def test_x_l2_persist_flag_rules():
     assert N.nest_batched_matvec_f32(ctypes.byref(d), 1, 64, 64, None, None, None, None) == N.NEST_ERR_INVALID_ARG
     assert N.nest_nested_stencil_f64(ctypes.byref(d), 1, 4, None, None, None, None, None, None) == \
         N.NEST_ERR_INVALID_ARG
-    with pytest.raises(P.NestError) as e:   # the x ring: unsupported
-        P.spmv_plan(1000, 1000, 8000, simdlen=2, x_halo=64, threads_per_team=256, x_l2_persist=True)
-    assert e.value.status == N.NEST_ERR_UNSUPPORTED and "x ring" in str(e.value)
     with pytest.raises(P.NestError) as e:   # the two-level teams-generic baseline: unsupported
         P.spmv_plan(1000, 1000, 8000, simdlen=1, mode="teams_generic", x_l2_persist=True)
     assert e.value.status == N.NEST_ERR_UNSUPPORTED

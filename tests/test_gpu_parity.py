@@ -671,6 +671,20 @@ def test_spmv_x_l2_persist_is_a_cache_policy_only(P, banded, cfg1, S):
                     assert_close(y1, yref, aref, 1e-12)
 
 
+def test_spmv_x_l2_persist_with_the_x_ring(P, banded):
+    # the x ring (shared staging of x) takes the window too: same bits
+    rp, col, val, x, yref, aref = banded["int"]
+    t = [dev(rp), dev(col), dev(val), dev(x)]
+    for S, vec, quad in ((2, True, False), (4, False, False), (2, True, True)):
+        cfg = dict(simdlen=S, x_halo=700, threads_per_team=768, vec128=vec, quad=quad)
+        y0 = host(P.spmv_csr_f64(*t, **cfg))
+        y1 = host(P.spmv_csr_f64(*t, x_l2_persist=True, **cfg))
+        assert np.array_equal(bits(y1), bits(y0)) and np.array_equal(bits(y1), bits(yref)), cfg
+    info = P.spmv_plan(rp.size - 1, x.size, val.size, simdlen=2, x_halo=700, threads_per_team=768,
+                       x_l2_persist=True)
+    assert info["kernel"] == 1 and info["l2_window_bytes"] == x.size * 8
+
+
 def test_spmv_x_l2_persist_plan_and_flush(P, banded):
     rp, col, val, x, yref, aref = banded["real"]
     n = rp.size - 1

@@ -62,6 +62,7 @@ def launch(draw):
     elif kind == "ring":
         cfg["x_halo"] = draw(st.sampled_from([1, 64, 700]))
         cfg["threads_per_team"] = max(64, cfg["threads_per_team"])
+        cfg["x_l2_persist"] = draw(st.booleans())
     else:
         cfg.update(blocked=draw(st.booleans()), x_l2_persist=kind == "persist")
     return cfg
