@@ -59,6 +59,8 @@ CONFIGS = {
                                                vec128=fl != "scalar", quad=fl == "quads", x_l2_persist=True))
                 for S in (2, 4, 8) for m in ("generic_smem", "generic_shfl") for fl in ("scalar", "pairs", "quads")
                 for T in (768, 1024)],
+    "ringp": [(f"ring S2 pairs T768 kb2{' persist' if pe else ''}", dict(simdlen=2, vec128=True, x_halo=4096,
+                teams_per_sm=2, outer_unroll=2, threads_per_team=768, x_l2_persist=pe)) for pe in (False, True)],
     "waves": [(f"S2 quads persist teams {nt}", dict(simdlen=2, quad=True, blocked=True, threads_per_team=1024,
                                                     x_l2_persist=True, num_teams=nt))
               for nt in (0, 592, 888, 1184, 2368, 4736)],
