@@ -435,6 +435,43 @@ nest_status nest_spmv_csr_f64_xpeer(const nest_desc *desc, nest_xpeer *xp, int64
                                     void *stream);
 nest_status nest_xpeer_destroy(nest_xpeer *xp);
 
+/* ---- NEXT-4b: symmetric x -- every rank's slice of x mapped into ONE virtual range ----
+ * The peer-gather SpMV above looks up the owner of each far column and loads that
+ * rank's slice pointer (a division and a dependent load per gather: +21-79% on one
+ * GPU, profiles/r02s3_x_l2_persist.md §12).  Here each rank's x slice is a CUDA
+ * virtual-memory allocation (cuMemCreate) exported as a POSIX file descriptor;
+ * every rank imports the others' descriptors and maps all slices back to back, so
+ * global column j is at nest_xsym_x(xs)[j] on every rank and the row-partitioned
+ * SpMV is the ordinary nest_spmv_csr_f64 on that pointer (rows = the rank's shard,
+ * 0-based rowptr, GLOBAL column indices; any variant), its remote columns read
+ * from the owners' memory over NVLink / NVSwitch.  Slices hold xchunk columns each,
+ * xchunk = ceil(ncols / nranks) rounded up to the allocation granularity (so the
+ * slices tile x exactly); rank r owns columns [r*xchunk, (r+1)*xchunk) and writes
+ * them through nest_xsym_local_x.  Ordering is the caller's: the writes of every
+ * rank's slice must complete (stream sync + a process barrier) before any rank's
+ * SpMV, and the SpMVs before a slice is rewritten.  Driver entry points are resolved
+ * at run time (NEST_ERR_UNSUPPORTED without them).
+ *   nest_xsym_create(nranks, rank, ncols, &xs, &fd): this rank's slice, its FD;
+ *   the caller passes every FD to every other rank (e.g. SCM_RIGHTS on a unix socket);
+ *   nest_xsym_open(xs, fds[nranks]): import and map (fds[rank] ignored; the caller
+ *   may close the received descriptors afterwards).
+ * nest_xsym_create_local: single process, nranks slices on the current device
+ * mapped the same way (tests, or one process driving several slices). */
+typedef struct nest_xsym nest_xsym;
+nest_status nest_xsym_create(int32_t nranks, int32_t rank, int64_t ncols_global, nest_xsym **out,
+                             int32_t *fd_out);
+nest_status nest_xsym_open(nest_xsym *xs, const int32_t *fds /* [nranks] */);
+nest_status nest_xsym_create_local(int32_t nranks, int64_t ncols_global, nest_xsym **out);
+/* The contiguous x (device pointer; NULL before open) and this rank's slice of it. */
+double *nest_xsym_x(nest_xsym *xs);
+double *nest_xsym_local_x(nest_xsym *xs);
+int64_t nest_xsym_xchunk(const nest_xsym *xs);
+/* Stream-ordered device-to-device copy of min(n, xchunk) doubles from src into rank
+ * `rank`'s slice (columns [rank*xchunk, ...)); multi-process form: the own rank only. */
+nest_status nest_xsym_set_x(nest_xsym *xs, int32_t rank, const double *src, int64_t n, void *stream);
+/* Synchronises the device, unmaps and releases. */
+nest_status nest_xsym_destroy(nest_xsym *xs);
+
 /* Release library-owned device scratch of the current device; if a
  * NEST_F_X_L2_PERSIST call raised the device's persisting-L2 limit, return the
  * persisting lines to normal and restore the limit it found. */

@@ -101,6 +101,14 @@ SIGNATURES = {
     "nest_spmv_csr_f64_xpeer": (_st, [_D, _vp, _i64, _i64, _i64, _vp, _vp, _vp, _vp, _vp]),
     "nest_xpeer_destroy": (_st, [_vp]),
     "nest_shutdown": (_st, []),
+    "nest_xsym_create": (_st, [_i32, _i32, _i64, ctypes.POINTER(ctypes.c_void_p), ctypes.POINTER(_i32)]),
+    "nest_xsym_open": (_st, [_vp, ctypes.POINTER(_i32)]),
+    "nest_xsym_create_local": (_st, [_i32, _i64, ctypes.POINTER(ctypes.c_void_p)]),
+    "nest_xsym_x": (_vp, [_vp]),
+    "nest_xsym_local_x": (_vp, [_vp]),
+    "nest_xsym_xchunk": (_i64, [_vp]),
+    "nest_xsym_set_x": (_st, [_vp, _i32, _vp, _i64, _vp]),
+    "nest_xsym_destroy": (_st, [_vp]),
 }
 
 for _name, (_res, _args) in SIGNATURES.items():

@@ -217,3 +217,117 @@ class XPeer:
             self.close()
         except Exception:
             pass
+
+
+def _exchange_fds(fd: int, rank: int, nranks: int, tag: str, group=None) -> list:
+    """Every rank's file descriptor to every rank (SCM_RIGHTS over unix sockets on this
+    node; torch.distributed only orders the steps).  Returns a list of nranks fds
+    (the entry at `rank` is `fd` itself)."""
+    import os
+    import socket
+    import threading
+
+    import torch.distributed as dist
+    path = lambda r: f"/tmp/nest_xsym_{tag}_{r}.sock"   # noqa: E731
+    me = path(rank)
+    if os.path.exists(me):
+        os.unlink(me)
+    srv = socket.socket(socket.AF_UNIX, socket.SOCK_STREAM)
+    srv.bind(me)
+    srv.listen(nranks)
+    got = {rank: fd}
+
+    def serve():
+        for _ in range(nranks - 1):
+            conn, _ = srv.accept()
+            with conn:
+                msg, fds, _, _ = socket.recv_fds(conn, 16, 1)
+                got[int(msg.decode())] = fds[0]
+    t = threading.Thread(target=serve, daemon=True)
+    t.start()
+    dist.barrier(group=group)                 # every rank listens
+    for r in range(nranks):
+        if r != rank:
+            with socket.socket(socket.AF_UNIX, socket.SOCK_STREAM) as c:
+                c.connect(path(r))
+                socket.send_fds(c, [str(rank).encode()], [fd])
+    t.join()
+    srv.close()
+    dist.barrier(group=group)                 # every rank has every descriptor
+    os.unlink(me)
+    return [got[r] for r in range(nranks)]
+
+
+class XSym:
+    """NEXT-4b: x as ONE virtual range over every rank's slice (CUDA virtual memory,
+    POSIX file descriptors exchanged on this node).  ``x`` is the contiguous global x
+    (column j at x[j] on every rank), so the row-partitioned SpMV is the ordinary
+    ``spmv_csr_f64(rowptr_local, colind_global, val, xs.x(), ...)`` -- any variant.
+    ``nranks`` without a process group: single-process form, every slice local."""
+
+    def __init__(self, ncols_global: int, group=None, *, nranks=None, tag="x"):
+        import os
+        torch = _torch()
+        self._torch = torch
+        self._h = ctypes.c_void_p()
+        self.ncols = int(ncols_global)
+        if nranks is not None:
+            self.nranks, self.rank = int(nranks), 0
+            check(N.nest_xsym_create_local(self.nranks, self.ncols, ctypes.byref(self._h)),
+                  "nest_xsym_create_local")
+            return
+        import torch.distributed as dist
+        self.rank, self.nranks = dist.get_rank(group), dist.get_world_size(group)
+        fd = ctypes.c_int32(-1)
+        check(N.nest_xsym_create(self.nranks, self.rank, self.ncols, ctypes.byref(self._h), ctypes.byref(fd)),
+              "nest_xsym_create")
+        fds = _exchange_fds(fd.value, self.rank, self.nranks, f"{tag}_{os.getppid()}", group)
+        arr = (ctypes.c_int32 * self.nranks)(*fds)
+        check(N.nest_xsym_open(self._h, arr), "nest_xsym_open")
+        for r, f in enumerate(fds):   # imported (or exported) allocations keep their own references
+            os.close(f)
+
+    @property
+    def xchunk(self) -> int:
+        return int(N.nest_xsym_xchunk(self._h))
+
+    def x_ptr(self) -> int:
+        return int(N.nest_xsym_x(self._h))
+
+    def local_x_ptr(self) -> int:
+        return int(N.nest_xsym_local_x(self._h))
+
+    def set_x(self, x_part, rank=None, stream=None):
+        """Copy the first min(len, xchunk) values of x_part (a CUDA tensor) into rank r's
+        slice, columns [r*xchunk, ...) (default: this rank's), stream-ordered."""
+        torch = self._torch
+        r = self.rank if rank is None else int(rank)
+        check(N.nest_xsym_set_x(self._h, r, _dev(x_part, torch.float64, None, "x_part"), x_part.numel(),
+                                _stream(stream)), "nest_xsym_set_x")
+
+    def spmv_csr_f64(self, rowptr, colind, val, y_local=None, *, stream=None, **cfg):
+        """y_local = A[local rows] @ x (global columns) on the symmetric x.  Ordering of
+        the slices' writes against this call is the caller's (sync + barrier)."""
+        torch = self._torch
+        nrows = rowptr.numel() - 1
+        nnz = val.numel()
+        if y_local is None:
+            y_local = torch.empty(nrows, dtype=torch.float64, device=val.device)
+        d = make_desc(**cfg)
+        check(N.nest_spmv_csr_f64(ctypes.byref(d), nrows, self.ncols, nnz,
+                                  _dev(rowptr, torch.int64, nrows + 1, "rowptr"),
+                                  _dev(colind, torch.int32, nnz, "colind"), _dev(val, torch.float64, nnz, "val"),
+                                  ctypes.c_void_p(self.x_ptr()), _dev(y_local, torch.float64, nrows, "y"),
+                                  _stream(stream)), "nest_spmv_csr_f64 (xsym)")
+        return y_local
+
+    def close(self):
+        if self._h:
+            check(N.nest_xsym_destroy(self._h), "nest_xsym_destroy")
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

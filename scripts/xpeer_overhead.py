@@ -2,7 +2,8 @@
 slices, the owner of column c = c / xchunk looked up per gather) against the plain
 kernel on the same rows with one x: the in-kernel cost of the owner lookup, without
 NVLink.  Rank 0's shard of configs[4] at P = 8 (12.5M rows, x = 800 MB).  Median of 10
-launches, L2 flushed before each (developer tool)."""
+launches, L2 flushed before each (developer tool).  Also the symmetric x (NEXT-4b):
+the same 8 slices mapped into one virtual range, plain kernel."""
 import os
 import statistics
 import sys
@@ -26,6 +27,12 @@ for r in range(nranks):
     b, k = P.local_x_range(spec.ncols, nranks, r)
     s[:k] = dx[b:b + k]
     sl.append(s)
+xsym = P.XSym(spec.ncols, nranks=nranks)   # the same slices, mapped into one virtual range
+for r in range(nranks):
+    lo = r * xsym.xchunk
+    if lo < spec.ncols:
+        xsym.set_x(dx[lo:lo + xsym.xchunk], rank=r)
+torch.cuda.synchronize()
 flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
 B = nnz * 12 + (nloc + 1) * 8 + nloc * 8 + spec.ncols * 8
 y = torch.empty(nloc, dtype=torch.float64, device="cuda")
@@ -35,10 +42,12 @@ for S, vec in ((8, True), (2, True), (8, False)):
     plain = lambda: P.spmv_csr_f64(drp, dcol, dval, dx, y, ncols=spec.ncols, **cfg)
     peer = lambda: xp.spmv_csr_f64(spec.nrows, drp, dcol, dval, y, **cfg)
     res = {}
-    for name, fn in (("plain x", plain), ("peer slices", peer)):
+    sym = lambda: xsym.spmv_csr_f64(drp, dcol, dval, y, **cfg)
+    for name, fn in (("plain x", plain), ("peer slices", peer), ("symmetric x", sym)):
         fn()
         ms = statistics.median(bench.time_steps(torch, fn, flush, P, 10))
         res[name] = ms
         print(f"S={S} {'pairs' if vec else 'scalar'} {name:12s} {ms:.4f} ms  {B / ms / 1e6:.0f} GB/s", flush=True)
     xp.close()
-    print(f"   owner-lookup overhead {res['peer slices'] / res['plain x'] - 1:+.1%}", flush=True)
+    print(f"   owner-lookup overhead {res['peer slices'] / res['plain x'] - 1:+.1%}, "
+          f"symmetric x {res['symmetric x'] / res['plain x'] - 1:+.1%}", flush=True)
