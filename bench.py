@@ -612,6 +612,21 @@ def run_gpu_multi(args, rank, world, local_rank):
         checks["peer_gather"] = parity(d_y.cpu().numpy(), yref, aref)
     except P.NestError as e:
         xp, xp_err = None, str(e)
+    # NEXT-4b: x as one virtual range over every rank's slice (CUDA virtual memory, file
+    # descriptors over a unix socket): the plain kernel on a contiguous x, remote columns
+    # read over NVLink; x written once (the timed step is the SpMV alone)
+    xsym_err = None
+    try:
+        xsym = P.XSym(spec.ncols, tag=f"bench{os.getppid()}")
+        lo = rank * xsym.xchunk
+        if lo < spec.ncols:
+            xsym.set_x(torch.from_numpy(x_full_host[lo:lo + xsym.xchunk].copy()).to(dev))
+        torch.cuda.synchronize()
+        dist.barrier()
+        res["step_symmetric_x"] = timed(lambda: xsym.spmv_csr_f64(drp, dcol, dval, d_y, **cfg), args.steps)
+        checks["symmetric_x"] = parity(d_y.cpu().numpy(), yref, aref)
+    except P.NestError as e:
+        xsym, xsym_err = None, str(e)
     head = "step_allgather_spmv" if "step_allgather_spmv" in res else "step_peer_gather"
     ms, clocks = res[head]
     worst = maxr(max(c["worst_rel_to_abs"] for c in checks.values()))
@@ -646,7 +661,7 @@ def run_gpu_multi(args, rank, world, local_rank):
                                         if "allgather_alone" in res else None),
                 "parity": {"rows_checked": spec.nrows, "worst_rel_to_abs_over_ranks": worst,
                            "ok": bool(worst <= 1e-12), "per_variant_rank0": checks},
-                "xpeer_error": xp_err,
+                "xpeer_error": xp_err, "xsym_error": xsym_err,
                 "gpu_launches": args.steps * (3 if head == "step_allgather_spmv" else 5),
                 "gpu_launches_detail": ("per step: NCCL all-gather + SpMV kernel (+ 2 l2_flush kernels outside "
                                         "the events)" if head == "step_allgather_spmv" else
@@ -662,6 +677,8 @@ def run_gpu_multi(args, rank, world, local_rank):
         print(json.dumps(line), flush=True)
     if xp is not None:
         xp.close()
+    if xsym is not None:
+        xsym.close()
     if comm is not None:
         comm.close()
 
