@@ -190,3 +190,28 @@ def test_xpeer_random_virtual_ranks(P, m, nranks, S, mode, vec, blocked):
         finally:
             xp.close()
         assert np.array_equal(bits(y.cpu().numpy()), bits(yref[rb:rb + nloc])), (nranks, r, S, mode, vec)
+
+
+@settings(max_examples=80, deadline=None, derandomize=True)
+@given(int_csr(), st.integers(1, 8), launch())
+def test_xsym_random_virtual_ranks(P, m, nranks, cfg):
+    # NEXT-4b: every shard's rows on the symmetric x (any variant), bit-exact vs the oracle
+    rp, col, val, x = m
+    n = rp.size - 1
+    yref, _ = oracle.spmv_csr_f64(rp, col, val, x)
+    xs = P.XSym(x.size, nranks=nranks)
+    try:
+        for r in range(nranks):
+            lo = r * xs.xchunk
+            if lo < x.size:
+                xs.set_x(torch.from_numpy(x[lo:lo + xs.xchunk].copy()).cuda(), rank=r)
+        torch.cuda.synchronize()
+        for r in range(nranks):
+            _, rb, nloc = P.shard_rows(n, nranks, r)
+            lrp = rp[rb:rb + nloc + 1] - rp[rb]
+            t = [torch.from_numpy(np.ascontiguousarray(a)).cuda()
+                 for a in (lrp, col[rp[rb]:rp[rb + nloc]], val[rp[rb]:rp[rb + nloc]])]
+            y = _run(P, lambda: xs.spmv_csr_f64(*t, **cfg))
+            assert np.array_equal(bits(y.cpu().numpy()), bits(yref[rb:rb + nloc])), (nranks, r, cfg)
+    finally:
+        xs.close()
