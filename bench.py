@@ -610,8 +610,8 @@ def run_gpu_multi(args, rank, world, local_rank):
         res["step_peer_gather"] = timed(lambda: xp.spmv_csr_f64(spec.nrows, drp, dcol, dval, d_y, **cfg),
                                         args.steps)
         checks["peer_gather"] = parity(d_y.cpu().numpy(), yref, aref)
-    except P.NestError as e:
-        xp, xp_err = None, str(e)
+    except Exception as e:   # an optional leg must not take the bench down
+        xp, xp_err = None, repr(e)
     # NEXT-4b: x as one virtual range over every rank's slice (CUDA virtual memory, file
     # descriptors over a unix socket): the plain kernel on a contiguous x, remote columns
     # read over NVLink; x written once (the timed step is the SpMV alone)
@@ -625,8 +625,8 @@ def run_gpu_multi(args, rank, world, local_rank):
         dist.barrier()
         res["step_symmetric_x"] = timed(lambda: xsym.spmv_csr_f64(drp, dcol, dval, d_y, **cfg), args.steps)
         checks["symmetric_x"] = parity(d_y.cpu().numpy(), yref, aref)
-    except P.NestError as e:
-        xsym, xsym_err = None, str(e)
+    except Exception as e:   # an optional leg must not take the bench down
+        xsym, xsym_err = None, repr(e)
     head = "step_allgather_spmv" if "step_allgather_spmv" in res else "step_peer_gather"
     ms, clocks = res[head]
     worst = maxr(max(c["worst_rel_to_abs"] for c in checks.values()))
