@@ -278,14 +278,28 @@ class XSym:
             return
         import torch.distributed as dist
         self.rank, self.nranks = dist.get_rank(group), dist.get_world_size(group)
+
+        def all_ok(status):   # every rank agrees before the next collective step
+            dev = "cuda" if dist.get_backend(group) == "nccl" else "cpu"
+            t = torch.tensor([1 if status == N.NEST_OK else 0], dtype=torch.int32, device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MIN, group=group)
+            return int(t.item()) == 1
+
         fd = ctypes.c_int32(-1)
-        check(N.nest_xsym_create(self.nranks, self.rank, self.ncols, ctypes.byref(self._h), ctypes.byref(fd)),
-              "nest_xsym_create")
+        st = N.nest_xsym_create(self.nranks, self.rank, self.ncols, ctypes.byref(self._h), ctypes.byref(fd))
+        if not all_ok(st):
+            if fd.value >= 0:
+                os.close(fd.value)
+            self.close()
+            check(st if st != N.NEST_OK else N.NEST_ERR_CUDA, "nest_xsym_create (on some rank)")
         fds = _exchange_fds(fd.value, self.rank, self.nranks, f"{tag}_{os.getppid()}", group)
         arr = (ctypes.c_int32 * self.nranks)(*fds)
-        check(N.nest_xsym_open(self._h, arr), "nest_xsym_open")
-        for r, f in enumerate(fds):   # imported (or exported) allocations keep their own references
+        st = N.nest_xsym_open(self._h, arr)
+        for f in fds:   # the imported (or exported) allocations keep their own references
             os.close(f)
+        if not all_ok(st):
+            self.close()
+            check(st if st != N.NEST_OK else N.NEST_ERR_CUDA, "nest_xsym_open (on some rank)")
 
     @property
     def xchunk(self) -> int:
