@@ -70,3 +70,43 @@ def test_row_partitioned_spmv_gloo(world):
         assert nfull == world * -(-spec.ncols // world)
         y = np.concatenate([y for _, y in sorted(ys, key=lambda t: t[0])])
         assert np.array_equal(y.view(np.int64), yref.view(np.int64))
+
+
+def _fd_worker(rank, world, port, tmpdir, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        from paper_conf_icpp_wrightdtcc23_b200.dist import _exchange_fds
+        # each rank opens its own file holding its rank number and passes the descriptor
+        path = os.path.join(tmpdir, f"r{rank}")
+        with open(path, "w") as f:
+            f.write(f"rank {rank}")
+        fd = os.open(path, os.O_RDONLY)
+        fds = _exchange_fds(fd, rank, world, f"gloo{port}")
+        got = []
+        for r, f in enumerate(fds):
+            os.lseek(f, 0, os.SEEK_SET)
+            got.append(os.read(f, 64).decode())
+            os.close(f)
+        q.put((rank, got))
+    except Exception as e:
+        q.put((rank, repr(e)))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_symmetric_x_fd_exchange_gloo(world, tmp_path):
+    # NEXT-4b host logic: every rank receives every other rank's file descriptor (SCM_RIGHTS
+    # over unix sockets, ordered by the process group) and it refers to the sender's object
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_fd_worker, args=(r, world, port, str(tmp_path), q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = dict(q.get(timeout=120) for _ in procs)
+    for p in procs:
+        p.join(timeout=30)
+    for r in range(world):
+        assert res[r] == [f"rank {k}" for k in range(world)], res
