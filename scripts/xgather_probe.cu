@@ -596,7 +596,7 @@ __global__ void __launch_bounds__(TB, MINB)
 // Per-team start / end times (%globaltimer, ns) of the headline structure: how much of the
 // kernel is the tail after the median team has finished?
 __device__ unsigned long long g_t0[1024], g_t1[1024];
-template <int S>
+template <int S, bool REV = false>
 __global__ void __launch_bounds__(1024, 2)
     spmv_qt(const int64_t* __restrict__ rp, const int* __restrict__ col, const double* __restrict__ val,
             const double* __restrict__ x, double* __restrict__ y, int n, int chunk, int nnz) {
@@ -607,7 +607,7 @@ __global__ void __launch_bounds__(1024, 2)
     }
     const int G = blockDim.x / S;
     const int g = threadIdx.x / S, lane = threadIdx.x % S;
-    const int cs = blockIdx.x * chunk;
+    const int cs = (REV ? gridDim.x - 1 - blockIdx.x : blockIdx.x) * chunk;
     const int ce = min(n, cs + chunk);
     for (int i = cs + g; i < ce; i += G) {
         const int b = (int)__ldg(rp + i), e = (int)__ldg(rp + i + 1);
@@ -809,12 +809,8 @@ int main(int argc, char** argv) {
         int rows_per_team = 0;   // > 0: non-persistent grid of ceil(n / rows_per_team) teams
     } vs[] = {
         {"S2 quads ldg (headline)", spmv_q<2, 0>, 1024, 0, "q"},
-        {"S2 quads apw 63MB", spmv_q<2, 0>, 1024, 0, nullptr, 63},
-        {"stagediag S2 far 2x1024", spmv_stagediag<2, 1, 1024, 1>, 1024, 114688, nullptr, 63},
-        {"stagediag S2 far 1x1024 (216KB)", spmv_stagediag<2, 1, 1024, 1>, 1024, 221184, nullptr, 63},
-        {"stagediag S2 far 1x1024 rounds", spmv_stagediag<2, 1, 1024, 1, true>, 1024, 221184, nullptr, 63},
-        {"stagediag S2 far 2x1024 rounds", spmv_stagediag<2, 1, 1024, 1, true>, 1024, 114688, nullptr, 63},
-        {"stagediag S2 nofar 1x1024 rounds", spmv_stagediag<2, 0, 1024, 1, true>, 1024, 221184, nullptr, 63},
+        {"S2 quads timed teams", spmv_qt<2>, 1024, 0, nullptr, 0},
+        {"S2 quads timed teams apw", spmv_qt<2>, 1024, 0, nullptr, 63},
     };
     int k = 0;
     for (auto& v : vs) {
@@ -887,7 +883,9 @@ int main(int argc, char** argv) {
             std::sort(st.begin(), st.end());
             std::sort(en.begin(), en.end());
             if (getenv("XG_DUMP")) {
-                FILE* f = fopen(getenv("XG_DUMP"), "w");
+                char fn[512];
+                snprintf(fn, sizeof fn, "%s_%d.txt", getenv("XG_DUMP"), k);
+                FILE* f = fopen(fn, "w");
                 for (int q = 0; q < grid; ++q) fprintf(f, "%d %.2f %.2f\n", q, (t0[q] - base) * 1e-3, (t1[q] - base) * 1e-3);
                 fclose(f);
             }
