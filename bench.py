@@ -270,6 +270,10 @@ HEADLINE = (2, "spmd", 1, 1024, 0, "bqp")
 SIMDLEN1 = [c for c in CANDIDATES if c[0] == 1]
 # configs[4] (16 nnz/row): wider groups pay (DESIGN.md Fig 9 analogue / cfg5 table)
 HEADLINE_CFG5 = (8, "spmd", 1, 1024, 0, "bv")
+# the local SpMV of a rank's configs[4] shard at N > 1: fastest per shard size on one B200
+# (profiles/r02s3/shard_configs.txt: S = 8 quads at N = 2, S = 4 quads from N = 4 on)
+SHARD_HEADLINE = {2: (8, "spmd", 1, 1024, 0, "bq")}
+SHARD_HEADLINE_DEFAULT = (4, "spmd", 1, 1024, 0, "bq")
 
 
 def cfg_of(c):
@@ -573,7 +577,8 @@ def run_gpu_multi(args, rank, world, local_rank):
     dist.all_reduce(nnz_t)
     B = alg_bytes(spec.nrows, spec.ncols, int(nnz_t.item()))
     B_local = nnz * 12 + (nloc + 1) * 8 + nloc * 8 + spec.ncols * 8
-    cfg = cfg_of(HEADLINE_CFG5)
+    local_c = SHARD_HEADLINE.get(world, SHARD_HEADLINE_DEFAULT)
+    cfg = cfg_of(local_c)
 
     def maxr(v):
         tt = torch.tensor([v], dtype=torch.float64, device=dev if not SHARE_GPU else "cpu")
@@ -604,10 +609,11 @@ def run_gpu_multi(args, rank, world, local_rank):
         res["local_spmv_alone"] = timed(lambda: P.spmv_csr_f64(drp, dcol, dval, d_xf, d_y, ncols=spec.ncols,
                                                                **cfg), args.steps)
     xp_err = None
+    cfg_xp = dict(cfg, quad=False)   # the peer-gather kernel takes scalar or pair loads
     try:
         xp = P.XPeer(spec.ncols)
         xp.set_local_x(d_xl)
-        res["step_peer_gather"] = timed(lambda: xp.spmv_csr_f64(spec.nrows, drp, dcol, dval, d_y, **cfg),
+        res["step_peer_gather"] = timed(lambda: xp.spmv_csr_f64(spec.nrows, drp, dcol, dval, d_y, **cfg_xp),
                                         args.steps)
         checks["peer_gather"] = parity(d_y.cpu().numpy(), yref, aref)
     except Exception as e:   # an optional leg must not take the bench down
@@ -627,7 +633,7 @@ def run_gpu_multi(args, rank, world, local_rank):
         checks["symmetric_x"] = parity(d_y.cpu().numpy(), yref, aref)
     except Exception as e:   # an optional leg must not take the bench down
         xsym, xsym_err = None, repr(e)
-    head = "step_allgather_spmv" if "step_allgather_spmv" in res else "step_peer_gather"
+    head = next(k for k in ("step_allgather_spmv", "step_symmetric_x", "step_peer_gather") if k in res)
     ms, clocks = res[head]
     worst = maxr(max(c["worst_rel_to_abs"] for c in checks.values()))
 
@@ -662,15 +668,16 @@ def run_gpu_multi(args, rank, world, local_rank):
                 "parity": {"rows_checked": spec.nrows, "worst_rel_to_abs_over_ranks": worst,
                            "ok": bool(worst <= 1e-12), "per_variant_rank0": checks},
                 "xpeer_error": xp_err, "xsym_error": xsym_err,
-                "gpu_launches": args.steps * (3 if head == "step_allgather_spmv" else 5),
-                "gpu_launches_detail": ("per step: NCCL all-gather + SpMV kernel (+ 2 l2_flush kernels outside "
-                                        "the events)" if head == "step_allgather_spmv" else
-                                        "per step: barrier + SpMV + barrier (+ 2 l2_flush)"),
+                "gpu_launches": args.steps * (5 if head == "step_peer_gather" else 3),
+                "gpu_launches_detail": {"step_allgather_spmv": "per step: NCCL all-gather (NCCL's kernel) + our SpMV "
+                                                               "kernel + 2 l2_flush kernels (outside the events)",
+                                        "step_symmetric_x": "per step: the SpMV kernel on the symmetric x + 2 l2_flush",
+                                        "step_peer_gather": "per step: barrier + SpMV + barrier + 2 l2_flush"}[head],
                 "clocks": clocks, "e2e": e2e}
         per_gpu = line["value"] / world
         line["roofline"] = {"bound": "hbm", "achieved": per_gpu, "peak": peak, "unit": "GB/s",
                             "frac": per_gpu / peak, "traffic": None, "peak_source": peak_src,
-                            "kernel": kernel_name(HEADLINE_CFG5),
+                            "kernel": kernel_name(local_c),
                             "note": "per GPU: algorithmic bytes of all ranks / world / max-over-ranks step time"}
         if not args.no_cpu_baseline:
             line["cpu_baseline"] = cpu_sample_multi(spec)
