@@ -119,19 +119,37 @@ static nest_status xsym_plan(int32_t nranks, int32_t rank, int64_t ncols, bool e
 static nest_status xsym_map(nest_xsym* xs) {
     const size_t total = xs->slice_bytes * (size_t)xs->nranks;
     CUresult r = drv().reserve(&xs->base, total, xs->gran, 0, 0);   // alignment: a power of two
-    if (r != CUDA_SUCCESS) return cu_fail(r, "cuMemAddressReserve");
-    for (int32_t q = 0; q < xs->nranks; ++q) {
-        r = drv().map(xs->base + (CUdeviceptr)(xs->slice_bytes * (size_t)q), xs->slice_bytes, 0, xs->handles[q], 0);
-        if (r != CUDA_SUCCESS) return cu_fail(r, "cuMemMap");
+    if (r != CUDA_SUCCESS) {
+        xs->base = 0;
+        return cu_fail(r, "cuMemAddressReserve");
     }
-    CUmemAccessDesc acc = {};
-    acc.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
-    acc.location.id = xs->dev;
-    acc.flags = CU_MEM_ACCESS_FLAGS_PROT_READWRITE;
-    r = drv().set_access(xs->base, total, &acc, 1);
-    if (r != CUDA_SUCCESS) return cu_fail(r, "cuMemSetAccess");
-    xs->mapped = true;
-    return NEST_OK;
+    int32_t done = 0;
+    const char* what = nullptr;
+    for (; done < xs->nranks; ++done) {
+        r = drv().map(xs->base + (CUdeviceptr)(xs->slice_bytes * (size_t)done), xs->slice_bytes, 0,
+                      xs->handles[done], 0);
+        if (r != CUDA_SUCCESS) {
+            what = "cuMemMap";
+            break;
+        }
+    }
+    if (!what) {
+        CUmemAccessDesc acc = {};
+        acc.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+        acc.location.id = xs->dev;
+        acc.flags = CU_MEM_ACCESS_FLAGS_PROT_READWRITE;
+        r = drv().set_access(xs->base, total, &acc, 1);
+        if (r == CUDA_SUCCESS) {
+            xs->mapped = true;
+            return NEST_OK;
+        }
+        what = "cuMemSetAccess";
+    }
+    // undo: the slices mapped so far, then the reservation (destroy then only releases handles)
+    for (int32_t q = 0; q < done; ++q) drv().unmap(xs->base + (CUdeviceptr)(xs->slice_bytes * (size_t)q), xs->slice_bytes);
+    drv().addr_free(xs->base, total);
+    xs->base = 0;
+    return cu_fail(r, what);
 }
 
 NEST_API nest_status nest_xsym_destroy(nest_xsym* xs) {
